@@ -1,0 +1,196 @@
+/*
+ * caqr.h -- C ABI of libcaqr.so: B200-native (sm_100a) TSQR / CAQR.
+ *
+ * Paper: M. Anderson, G. Ballard, J. Demmel, K. Keutzer, "Communication-Avoiding
+ * QR Decomposition for GPUs", IPDPS 2011.  "P:Lnnn" below = line nnn of the
+ * paper text, with its section.
+ *
+ * Operation (Sec. I): A = Q R with Q orthogonal (m x m) and R upper
+ * triangular (n x n), for a real m x n matrix A with m >= n, in single precision
+ * as the paper (Sec. IV) and in double precision.
+ *
+ * Method: TSQR panel factorisation (Sec. II.B, Fig. 2) -- the rows of
+ * a panel are cut into leaves, each leaf is QR-factored by Householder
+ * reflectors (kernel "factor"), the leaves' R factors are reduced
+ * pairwise up a binary tree of structured stacked-triangle QRs (kernel
+ * "factor_tree"; tree shape free) -- and, when n is
+ * wider than one panel, CAQR (Sec. II.C, Fig. 3/4): the panel's
+ * implicit Q^T is applied to the trailing columns leaf by leaf ("apply_qt_h",
+ * P:L665-668) and node by node up the tree ("apply_qt_tree"), then
+ * the grid is redrawn nb rows lower.  Reflectors are applied in
+ * compact-WY form I - V T V^T (Sec. II.A) with T built from the
+ * inner products of the vectors.
+ *
+ * Conventions for every entry point:
+ *   - Matrices are column-major with a leading dimension ("originally
+ *     stored in column major order").  ALL matrix and workspace pointers are
+ *     DEVICE pointers (cudaMalloc'd or torch CUDA storage) on the current device.
+ *   - Calls only enqueue work on `stream` (0 = legacy default stream); they never
+ *     synchronise the device, never allocate device memory, and are safe to
+ *     capture into a CUDA graph.  They are reentrant; the only process state is
+ *     a lazily-filled per-device attribute cache.
+ *   - Return value: LAPACK "info".  0 = success; -i = argument i is illegal (the
+ *     call does nothing); CAQR_ERR_CUDA (1) = a CUDA launch failed (see
+ *     caqr_last_cuda_error); CAQR_ERR_NCCL (2) = an NCCL call failed.
+ *     m = 0 or n = 0 is a quick return with 0.  NaN/Inf are not checked; they
+ *     propagate as in LAPACK.
+ *   - Householder convention (reading S1): LAPACK xLARFG
+ *     (beta = -sign(alpha)||x||, v(head) = 1, tau = (beta-alpha)/beta).  R_jj may be
+ *     negative; the library does not normalise signs.
+ *   - Rows n..m-1 of Q^T C depend on the tree shape and leaf size (several
+ *     correct answers, reading S17); rows 0..n-1 and every column norm
+ *     do not.
+ *   - `opts` selects the plan (leaf height, panel-group width).  NULL = the
+ *     default plan for (m, n, dtype).  The SAME opts must be passed to
+ *     caqr_workspace_bytes, caqr_factor_* and every later apply/form_q call on
+ *     that factorisation.
+ */
+#ifndef CAQR_H
+#define CAQR_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st *caqr_stream_t; /* == cudaStream_t */
+
+enum { CAQR_F32 = 0, CAQR_F64 = 1 };
+enum { CAQR_OK = 0, CAQR_ERR_CUDA = 1, CAQR_ERR_NCCL = 2, CAQR_ERR_UNSUPPORTED = 3 };
+
+/* Plan options; a field <= 0 means "default".
+ *   leaf_rows  b: rows per TSQR leaf (P:L633 / P:L822-823 used 64 and 128 on
+ *              Fermi; here a multiple of 32, b >= the panel-group width,
+ *              b <= 256).  Default 256.
+ *   panel_cols nb: CAQR panel-group width (one TSQR per group).
+ *              Default: n if n <= 256 (one whole-width TSQR), else 64. */
+typedef struct caqr_opts {
+    int64_t leaf_rows;
+    int64_t panel_cols;
+    int64_t reserved[6];
+} caqr_opts;
+
+/* Bytes of device workspace the factorisation of an m x n matrix of `dtype`
+ * needs (the T factors of every compact-WY block).  Returns 0 on illegal
+ * arguments (m < 0, n < 0, n > m, bad dtype, bad opts). */
+size_t caqr_workspace_bytes(int64_t m, int64_t n, int dtype, const caqr_opts *opts);
+
+/* QR factorisation, SGEQRF semantics (Sec. V.C: "doesn't return Q
+ * explicitly, instead it returns an intermediate representation that can later
+ * be used to retrieve or apply Q").
+ *   m, n       matrix size, m >= n >= 0                        (info -1, -2)
+ *   A          device, m x n, lda >= max(1,m); overwritten      (info -3, -4)
+ *              by the implicit-Q representation (Householder vectors of the
+ *              leaves below the leaves' diagonals, tree vectors in the upper
+ *              triangles of non-root leaf tops) and, in its top n x n upper
+ *              triangle, by R.
+ *   R          device, n x n, ldr >= max(1,n): receives R with  (info -5, -6)
+ *              the strict lower triangle zeroed.
+ *   ws         device workspace of ws_bytes >=                  (info -7, -8)
+ *              caqr_workspace_bytes(m, n, dtype, opts); receives the T factors.
+ *   opts       plan (may be NULL)                               (info -9)
+ *   stream     CUDA stream.
+ * A and ws together are the implicit Q; keep them unchanged for
+ * caqr_apply_qt / caqr_apply_q / caqr_form_q. */
+int caqr_factor_f32(int64_t m, int64_t n, float *A, int64_t lda, float *R, int64_t ldr,
+                    void *ws, size_t ws_bytes, const caqr_opts *opts, caqr_stream_t stream);
+int caqr_factor_f64(int64_t m, int64_t n, double *A, int64_t lda, double *R, int64_t ldr,
+                    void *ws, size_t ws_bytes, const caqr_opts *opts, caqr_stream_t stream);
+
+/* C <- Q^T C  (the trailing-matrix update of P:L603-610 applied to any C).
+ *   m, n, A, lda, ws, opts : exactly as passed to caqr_factor_*   (info -1..-4, -5)
+ *   k          columns of C, k >= 0                               (info -6)
+ *   C          device, m x k, ldc >= max(1,m), updated in place   (info -7, -8)
+ * Order: leaves, then the tree bottom-up (Fig. 4). */
+int caqr_apply_qt_f32(int64_t m, int64_t n, const float *A, int64_t lda, const void *ws,
+                      int64_t k, float *C, int64_t ldc, const caqr_opts *opts,
+                      caqr_stream_t stream);
+int caqr_apply_qt_f64(int64_t m, int64_t n, const double *A, int64_t lda, const void *ws,
+                      int64_t k, double *C, int64_t ldc, const caqr_opts *opts,
+                      caqr_stream_t stream);
+
+/* C <- Q C (tree top-down, then leaves).  Arguments as caqr_apply_qt_*. */
+int caqr_apply_q_f32(int64_t m, int64_t n, const float *A, int64_t lda, const void *ws,
+                     int64_t k, float *C, int64_t ldc, const caqr_opts *opts,
+                     caqr_stream_t stream);
+int caqr_apply_q_f64(int64_t m, int64_t n, const double *A, int64_t lda, const void *ws,
+                     int64_t k, double *C, int64_t ldc, const caqr_opts *opts,
+                     caqr_stream_t stream);
+
+/* Explicit thin Q (m x n) with A_original = Q R: SORGQR via CAQR (P:L905-910,
+ * "retrieving Q explicitly (SORGQR) using CAQR is just as efficient as
+ * factoring").  Q = (Q_leaves Q_tree) [I_n; 0].
+ *   m, n, A, lda, ws, opts : as passed to caqr_factor_*     (info -1..-5)
+ *   Q          device, m x n, ldq >= max(1,m); overwritten    (info -6, -7) */
+int caqr_form_q_f32(int64_t m, int64_t n, const float *A, int64_t lda, const void *ws,
+                    float *Q, int64_t ldq, const caqr_opts *opts, caqr_stream_t stream);
+int caqr_form_q_f64(int64_t m, int64_t n, const double *A, int64_t lda, const void *ws,
+                    double *Q, int64_t ldq, const caqr_opts *opts, caqr_stream_t stream);
+
+/* ---- Combine: the extra tree level of a row-sharded (multi-GPU) TSQR --------
+ * Not in the paper (single GPU); it is the distributed TSQR the
+ * paper cites, one more tree level whose leaves are GPUs.
+ * Rstack holds P n x n upper-triangular factors stacked vertically (a
+ * (P*n) x n column-major matrix, ld >= P*n; entries below each diagonal are
+ * ignored).  Factors the stack with the same structured binary tree as
+ * caqr_factor (deterministic: bitwise-identical results on every rank that
+ * passes the same stack), leaves the tree vectors in Rstack and the T factors
+ * in ws, writes the combined R (strict lower zeroed) to R.
+ *   P >= 1 (info -1), 0 <= n <= 256 (-2), Rstack/ld (-3, -4), R/ldr (-5, -6),
+ *   ws/ws_bytes (-7, -8) with ws_bytes >= caqr_combine_workspace_bytes. */
+size_t caqr_combine_workspace_bytes(int P, int64_t n, int dtype);
+int caqr_combine_f32(int P, int64_t n, float *Rstack, int64_t ld, float *R, int64_t ldr,
+                     void *ws, size_t ws_bytes, caqr_stream_t stream);
+int caqr_combine_f64(int P, int64_t n, double *Rstack, int64_t ld, double *R, int64_t ldr,
+                     void *ws, size_t ws_bytes, caqr_stream_t stream);
+/* C (P*n x k, ld ldc) <- Qc^T C (trans = 1) or Qc C (trans = 0), Qc the
+ * combine's orthogonal factor as left in Rstack/ws by caqr_combine_*. */
+int caqr_combine_apply_f32(int P, int64_t n, const float *Rstack, int64_t ld, const void *ws,
+                           int trans, int64_t k, float *C, int64_t ldc, caqr_stream_t stream);
+int caqr_combine_apply_f64(int P, int64_t n, const double *Rstack, int64_t ld, const void *ws,
+                           int trans, int64_t k, double *C, int64_t ldc, caqr_stream_t stream);
+
+/* ---- Multi-GPU row-sharded TSQR over NCCL (one process per GPU) -----------
+ * caqr_dist_create: nccl_unique_id = the 128-byte ncclUniqueId made by rank 0
+ * and broadcast by the caller (e.g. through torch.distributed).  The handle owns
+ * an NCCL communicator; the caller's current device is the rank's GPU.
+ * Returns 0 or CAQR_ERR_NCCL / -1 (nranks < 1) / -2 (rank out of range) /
+ * -3 (null pointers). */
+typedef struct caqr_dist caqr_dist;
+/* ncclGetUniqueId: writes the 128-byte id to out128 (host memory).  0 or
+ * CAQR_ERR_NCCL, -1 if out128 is NULL.  Call on rank 0 only. */
+int caqr_dist_unique_id(void *out128);
+int caqr_dist_create(caqr_dist **handle, int nranks, int rank, const void *nccl_unique_id);
+void caqr_dist_destroy(caqr_dist *handle);
+/* Every rank: local TSQR of its m_local x n shard (m_local >= n), ncclAllGather
+ * of the local R factors over NVLink, then the same deterministic combine on
+ * every rank -> the global R (identical bits on all ranks).
+ *   A, lda, ws, ws_bytes: the local factorisation (caqr_workspace_bytes(m_local,
+ *   n, dtype, opts));  gather: device, (nranks*n) x n, ld nranks*n, receives the
+ *   stacked local R's and then the combine's tree vectors;  cws, cws_bytes:
+ *   caqr_combine_workspace_bytes(nranks, n, dtype). */
+int caqr_dist_factor_f32(caqr_dist *h, int64_t m_local, int64_t n, float *A, int64_t lda,
+                         float *R, int64_t ldr, void *ws, size_t ws_bytes, float *gather,
+                         void *cws, size_t cws_bytes, const caqr_opts *opts,
+                         caqr_stream_t stream);
+int caqr_dist_factor_f64(caqr_dist *h, int64_t m_local, int64_t n, double *A, int64_t lda,
+                         double *R, int64_t ldr, void *ws, size_t ws_bytes, double *gather,
+                         void *cws, size_t cws_bytes, const caqr_opts *opts,
+                         caqr_stream_t stream);
+
+/* Diagnostics. */
+const char *caqr_strerror(int info);
+int caqr_last_cuda_error(void);          /* cudaError_t of the last CAQR_ERR_CUDA (thread-local) */
+const char *caqr_build_info(void);       /* "sm_100a ..." */
+/* Plan introspection (host only; for tests and the bench's roofline bookkeeping).
+ * Fills out[0..7] = {leaf_rows, panel_cols, groups, leaves(group 0),
+ * tree_levels(group 0), panels(group 0), kernel_launches(factor), 0}.
+ * Returns 0 or a negative info. */
+int caqr_plan_info(int64_t m, int64_t n, int dtype, const caqr_opts *opts, int64_t out[8]);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CAQR_H */

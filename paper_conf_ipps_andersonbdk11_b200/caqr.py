@@ -1,0 +1,291 @@
+"""Thin Python binding of libcaqr.so (include/caqr.h): argument marshalling only.
+
+Every step of the factorisation runs in the CUDA kernels behind the C ABI; this
+module only turns torch CUDA tensors into (pointer, leading dimension) pairs,
+picks the f32/f64 entry point, and raises on a nonzero LAPACK-style info.
+There is NO CPU fallback: without the built library or a GPU, calls raise.
+
+Matrices are column-major, as in the ABI: a torch tensor of shape (m, n) with
+stride (1, ld), ld >= m -- e.g. ``colmajor_empty(m, n)`` or ``x.t().contiguous().t()``.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import re
+import threading
+from typing import Optional, Tuple
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libcaqr.so")
+HEADER_PATH = os.path.join(os.path.dirname(_HERE), "include", "caqr.h")
+
+CAQR_F32, CAQR_F64 = 0, 1
+_lock = threading.Lock()
+_lib = None
+
+
+class CaqrError(RuntimeError):
+    def __init__(self, fn: str, info: int, msg: str = ""):
+        super().__init__(f"{fn} returned info={info}: {msg}")
+        self.info = info
+
+
+class Opts(ctypes.Structure):
+    """caqr_opts: leaf_rows (b), panel_cols (nb); 0 = default."""
+
+    _fields_ = [("leaf_rows", ctypes.c_int64), ("panel_cols", ctypes.c_int64),
+                ("reserved", ctypes.c_int64 * 6)]
+
+
+def _i64(*xs):
+    return [ctypes.c_int64] * len(xs)
+
+
+def lib() -> ctypes.CDLL:
+    """Load the in-tree libcaqr.so (raises if it was not built)."""
+    global _lib
+    with _lock:
+        if _lib is not None:
+            return _lib
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} missing: run `python -m paper_conf_ipps_andersonbdk11_b200.build` "
+                               "(no CPU fallback exists)")
+        L = ctypes.CDLL(LIB_PATH)
+        i64, vp, sz, ip = ctypes.c_int64, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int
+        op = ctypes.POINTER(Opts)
+        L.caqr_workspace_bytes.argtypes = [i64, i64, ip, op]
+        L.caqr_workspace_bytes.restype = sz
+        for suf in ("f32", "f64"):
+            f = getattr(L, f"caqr_factor_{suf}")
+            f.argtypes = [i64, i64, vp, i64, vp, i64, vp, sz, op, vp]
+            f.restype = ip
+            for name in ("apply_qt", "apply_q"):
+                f = getattr(L, f"caqr_{name}_{suf}")
+                f.argtypes = [i64, i64, vp, i64, vp, i64, vp, i64, op, vp]
+                f.restype = ip
+            f = getattr(L, f"caqr_form_q_{suf}")
+            f.argtypes = [i64, i64, vp, i64, vp, vp, i64, op, vp]
+            f.restype = ip
+            f = getattr(L, f"caqr_combine_{suf}")
+            f.argtypes = [ip, i64, vp, i64, vp, i64, vp, sz, vp]
+            f.restype = ip
+            f = getattr(L, f"caqr_combine_apply_{suf}")
+            f.argtypes = [ip, i64, vp, i64, vp, ip, i64, vp, i64, vp]
+            f.restype = ip
+            f = getattr(L, f"caqr_dist_factor_{suf}")
+            f.argtypes = [vp, i64, i64, vp, i64, vp, i64, vp, sz, vp, vp, sz, op, vp]
+            f.restype = ip
+        L.caqr_combine_workspace_bytes.argtypes = [ip, i64, ip]
+        L.caqr_combine_workspace_bytes.restype = sz
+        L.caqr_strerror.argtypes = [ip]
+        L.caqr_strerror.restype = ctypes.c_char_p
+        L.caqr_last_cuda_error.restype = ip
+        L.caqr_build_info.restype = ctypes.c_char_p
+        L.caqr_plan_info.argtypes = [i64, i64, ip, op, ctypes.POINTER(ctypes.c_int64)]
+        L.caqr_plan_info.restype = ip
+        L.caqr_dist_unique_id.argtypes = [vp]
+        L.caqr_dist_unique_id.restype = ip
+        L.caqr_dist_create.argtypes = [ctypes.POINTER(vp), ip, ip, vp]
+        L.caqr_dist_create.restype = ip
+        L.caqr_dist_destroy.argtypes = [vp]
+        L.caqr_dist_destroy.restype = None
+        _lib = L
+        return L
+
+
+def header_functions():
+    """Names of every function the C header declares (for the export test)."""
+    with open(HEADER_PATH) as f:
+        txt = f.read()
+    txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+    return sorted(set(re.findall(r"\b(caqr_[a-z0-9_]+)\s*\(", txt)))
+
+
+def make_opts(leaf_rows: int = 0, panel_cols: int = 0) -> Optional[Opts]:
+    if not leaf_rows and not panel_cols:
+        return None
+    return Opts(int(leaf_rows), int(panel_cols))
+
+
+def _optp(opts):
+    return ctypes.byref(opts) if opts is not None else None
+
+
+def _check(fn: str, info: int):
+    if info != 0:
+        L = lib()
+        msg = L.caqr_strerror(info).decode()
+        if info == 1:
+            msg += f" (cudaError {L.caqr_last_cuda_error()})"
+        raise CaqrError(fn, info, msg)
+
+
+# ---- torch plumbing ---------------------------------------------------------
+def _torch():
+    import torch
+
+    return torch
+
+
+def _dtype_code(t) -> Tuple[int, str]:
+    torch = _torch()
+    if t.dtype == torch.float32:
+        return CAQR_F32, "f32"
+    if t.dtype == torch.float64:
+        return CAQR_F64, "f64"
+    raise TypeError(f"caqr: dtype {t.dtype} not supported (float32 / float64)")
+
+
+def _colmajor(t, name: str):
+    if not t.is_cuda:
+        raise ValueError(f"caqr: {name} must be a CUDA tensor (no CPU path)")
+    if t.dim() != 2:
+        raise ValueError(f"caqr: {name} must be 2-D")
+    m, n = t.shape
+    if n > 1 and t.stride(0) != 1 and m > 1:
+        raise ValueError(f"caqr: {name} must be column-major (stride(0) == 1); use colmajor()")
+    ld = t.stride(1) if n > 1 else max(m, 1)
+    return t.data_ptr(), max(ld, m, 1)
+
+
+def colmajor_empty(m: int, n: int, dtype=None, device="cuda"):
+    torch = _torch()
+    return torch.empty((n, m), dtype=dtype or torch.float32, device=device).t()
+
+
+def colmajor(x):
+    """Column-major copy of a 2-D tensor (no copy if already column-major)."""
+    if x.dim() == 2 and (x.stride(0) == 1 or x.shape[1] <= 1):
+        return x
+    return x.t().contiguous().t()
+
+
+def _stream(stream):
+    torch = _torch()
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+# ---- the ABI, one Python function per C entry point (same names) ------------
+def caqr_workspace_bytes(m: int, n: int, dtype: int = CAQR_F32, opts: Optional[Opts] = None) -> int:
+    return int(lib().caqr_workspace_bytes(m, n, dtype, _optp(opts)))
+
+
+def caqr_plan_info(m: int, n: int, dtype: int = CAQR_F32, opts: Optional[Opts] = None) -> dict:
+    out = (ctypes.c_int64 * 8)()
+    _check("caqr_plan_info", lib().caqr_plan_info(m, n, dtype, _optp(opts), out))
+    keys = ["leaf_rows", "panel_cols", "groups", "leaves", "tree_levels", "panels", "launches"]
+    return {k: int(out[i]) for i, k in enumerate(keys)}
+
+
+def caqr_factor(A, R=None, ws=None, opts: Optional[Opts] = None, stream=None):
+    """Factor A in place (column-major CUDA tensor).  Returns (R, ws): R is n x n
+    (strict lower zero), ws the workspace holding T; A and ws are the implicit Q."""
+    torch = _torch()
+    code, suf = _dtype_code(A)
+    m, n = A.shape
+    pa, lda = _colmajor(A, "A")
+    if R is None:
+        R = colmajor_empty(n, n, A.dtype, A.device)
+    pr, ldr = _colmajor(R, "R")
+    need = caqr_workspace_bytes(m, n, code, opts)
+    if need == 0 and n > 0:
+        raise CaqrError("caqr_workspace_bytes", -2, "illegal size/opts")
+    if ws is None:
+        ws = torch.empty(max(need, 1), dtype=torch.uint8, device=A.device)
+    info = getattr(lib(), f"caqr_factor_{suf}")(m, n, pa, lda, pr, ldr, ws.data_ptr(), ws.numel(),
+                                                 _optp(opts), _stream(stream))
+    _check(f"caqr_factor_{suf}", info)
+    return R, ws
+
+
+def _apply(name, A, ws, C, n, opts, stream):
+    code, suf = _dtype_code(A)
+    m = A.shape[0]
+    pa, lda = _colmajor(A, "A")
+    pc, ldc = _colmajor(C, "C")
+    if C.shape[0] != m:
+        raise ValueError("C must have as many rows as A")
+    info = getattr(lib(), f"caqr_{name}_{suf}")(m, n, pa, lda, ws.data_ptr(), C.shape[1], pc, ldc,
+                                                 _optp(opts), _stream(stream))
+    _check(f"caqr_{name}_{suf}", info)
+    return C
+
+
+def caqr_apply_qt(A, ws, C, n=None, opts=None, stream=None):
+    """C <- Q^T C in place (A, ws as left by caqr_factor)."""
+    return _apply("apply_qt", A, ws, C, A.shape[1] if n is None else n, opts, stream)
+
+
+def caqr_apply_q(A, ws, C, n=None, opts=None, stream=None):
+    """C <- Q C in place."""
+    return _apply("apply_q", A, ws, C, A.shape[1] if n is None else n, opts, stream)
+
+
+def caqr_form_q(A, ws, Q=None, n=None, opts=None, stream=None):
+    """Explicit thin Q (m x n), A_original = Q R."""
+    code, suf = _dtype_code(A)
+    m = A.shape[0]
+    n = A.shape[1] if n is None else n
+    pa, lda = _colmajor(A, "A")
+    if Q is None:
+        Q = colmajor_empty(m, n, A.dtype, A.device)
+    pq, ldq = _colmajor(Q, "Q")
+    info = getattr(lib(), f"caqr_form_q_{suf}")(m, n, pa, lda, ws.data_ptr(), pq, ldq, _optp(opts),
+                                                 _stream(stream))
+    _check(f"caqr_form_q_{suf}", info)
+    return Q
+
+
+def caqr_combine_workspace_bytes(P: int, n: int, dtype: int = CAQR_F32) -> int:
+    return int(lib().caqr_combine_workspace_bytes(P, n, dtype))
+
+
+def caqr_combine(Rstack, P: int, R=None, ws=None, stream=None):
+    """Combine P stacked n x n R factors ((P*n) x n column-major, modified in
+    place) into one R.  Returns (R, ws)."""
+    torch = _torch()
+    code, suf = _dtype_code(Rstack)
+    n = Rstack.shape[1]
+    ps, ld = _colmajor(Rstack, "Rstack")
+    if R is None:
+        R = colmajor_empty(n, n, Rstack.dtype, Rstack.device)
+    pr, ldr = _colmajor(R, "R")
+    need = caqr_combine_workspace_bytes(P, n, code)
+    if ws is None:
+        ws = torch.empty(max(need, 1), dtype=torch.uint8, device=Rstack.device)
+    info = getattr(lib(), f"caqr_combine_{suf}")(P, n, ps, ld, pr, ldr, ws.data_ptr(), ws.numel(),
+                                                  _stream(stream))
+    _check(f"caqr_combine_{suf}", info)
+    return R, ws
+
+
+def caqr_combine_apply(Rstack, P: int, ws, C, trans: bool = True, stream=None):
+    code, suf = _dtype_code(Rstack)
+    n = Rstack.shape[1]
+    ps, ld = _colmajor(Rstack, "Rstack")
+    pc, ldc = _colmajor(C, "C")
+    info = getattr(lib(), f"caqr_combine_apply_{suf}")(P, n, ps, ld, ws.data_ptr(), int(trans),
+                                                        C.shape[1], pc, ldc, _stream(stream))
+    _check(f"caqr_combine_apply_{suf}", info)
+    return C
+
+
+def geqrf_flops(m: int, n: int) -> float:
+    """LAPACK count 2 m n^2 - 2 n^3 / 3 (the BASELINE metric's flop count)."""
+    return 2.0 * m * n * n - 2.0 * n ** 3 / 3.0
+
+
+def qr_host(A_host, opts=None, stream=None, pinned_out=None):
+    """End-to-end public call from host memory: H2D copy of A (pinned host
+    tensor, column-major), caqr_factor on the GPU, D2H copy of R.  Returns the
+    host R (and leaves the device factorisation in the returned tuple)."""
+    torch = _torch()
+    A_dev = colmajor_empty(A_host.shape[0], A_host.shape[1], A_host.dtype, "cuda")
+    A_dev.copy_(A_host, non_blocking=True)
+    R, ws = caqr_factor(A_dev, opts=opts, stream=stream)
+    out = pinned_out if pinned_out is not None else torch.empty(R.shape, dtype=R.dtype, pin_memory=True)
+    out.copy_(R, non_blocking=True)
+    return out, A_dev, ws

@@ -1,0 +1,472 @@
+// caqr.cu -- host planner + C ABI of libcaqr.so (declared in include/caqr.h).
+//
+// The host side is the paper's "CPU coordinates the GPU's actions and updates
+// pointers" (Sec. IV.B): it walks the plan -- panel groups, leaf
+// panels, tree levels (Fig. 4) -- and enqueues kernels on the
+// caller's stream.  No host synchronisation, no device allocation.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdint>
+#include <cstring>
+#include <mutex>
+
+#include "../../include/caqr.h"
+#include "tsqr_kernels.cuh"
+
+namespace caqr {
+
+static thread_local int g_last_cuda_error = 0;
+
+constexpr int64_t kMaxGroup = 256;  // widest single TSQR panel group
+constexpr int64_t kMaxLeaf = 256;   // tallest leaf the v1 kernels stage in shared memory
+
+struct Plan {
+    int64_t m = 0, n = 0;
+    int dtype = 0;
+    int64_t b = 0;   // leaf height
+    int64_t nb = 0;  // panel-group width
+    int64_t ngroups = 0;
+};
+
+static inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+static inline int64_t round_up(int64_t a, int64_t b) { return ceil_div(a, b) * b; }
+
+// Returns 0, or the info code of the offending argument position `opt_pos`.
+static int make_plan(int64_t m, int64_t n, int dtype, const caqr_opts* o, int opt_pos, Plan* pl) {
+    pl->m = m;
+    pl->n = n;
+    pl->dtype = dtype;
+    int64_t nb = (o && o->panel_cols > 0) ? o->panel_cols : (n <= kMaxGroup ? n : 64);
+    if (nb > kMaxGroup) return -opt_pos;
+    nb = std::max<int64_t>(1, std::min(nb, std::max<int64_t>(n, 1)));
+    int64_t b = (o && o->leaf_rows > 0) ? o->leaf_rows : kMaxLeaf;
+    if (b % 32 != 0 || b > kMaxLeaf) return -opt_pos;
+    b = std::max(b, round_up(nb, 32));
+    if (b > kMaxLeaf) return -opt_pos;
+    pl->nb = nb;
+    pl->b = b;
+    pl->ngroups = n == 0 ? 0 : ceil_div(n, nb);
+    return 0;
+}
+
+static Geom group_geom(const Plan& pl, int64_t g, int64_t lda) {
+    Geom G;
+    G.lda = lda;
+    G.col0 = g * pl.nb;
+    G.row0 = G.col0;
+    G.mrows = pl.m - G.row0;
+    G.ncols = (int32_t)std::min(pl.nb, pl.n - G.col0);
+    G.npan = (int32_t)ceil_div(G.ncols, kPW);
+    G.b = pl.b;
+    G.L = std::max<int64_t>(1, ceil_div(G.mrows, pl.b));
+    return G;
+}
+
+static inline int tree_levels(int64_t L) {
+    int lv = 0;
+    while ((int64_t(1) << lv) < L) ++lv;
+    return lv;
+}
+static inline int64_t merges_at(int64_t L, int level) {
+    const int64_t h = int64_t(1) << level;
+    return (L - 1 >= h) ? (L - 1 - h) / (2 * h) + 1 : 0;
+}
+static inline size_t group_t_elems(const Geom& G) { return (size_t)2 * G.L * G.npan * kPW * kPW; }
+
+static size_t plan_ws_bytes(const Plan& pl) {
+    size_t elems = 0;
+    for (int64_t g = 0; g < pl.ngroups; ++g) elems += group_t_elems(group_geom(pl, g, pl.m));
+    return elems * (pl.dtype == CAQR_F64 ? 8 : 4);
+}
+
+// ---- launch helpers ---------------------------------------------------------
+// Opt a kernel into > 48 KB of dynamic shared memory, once per (kernel, device).
+static cudaError_t allow_smem_ptr(const void* kernel, size_t bytes) {
+    if (bytes <= 48 * 1024) return cudaSuccess;
+    static std::mutex mu;
+    static const void* keys[256];
+    static int devs[256];
+    static int nkeys = 0;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    std::lock_guard<std::mutex> lk(mu);
+    for (int i = 0; i < nkeys; ++i)
+        if (keys[i] == kernel && devs[i] == dev) return cudaSuccess;
+    int optin = 0;
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    if ((size_t)optin < bytes) return cudaErrorInvalidValue;
+    cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, optin);
+    if (e == cudaSuccess && nkeys < 256) {
+        keys[nkeys] = kernel;
+        devs[nkeys] = dev;
+        ++nkeys;
+    }
+    return e;
+}
+template <typename K>
+static cudaError_t allow_smem(K kernel, size_t bytes) {
+    return allow_smem_ptr(reinterpret_cast<const void*>(kernel), bytes);
+}
+
+template <typename T>
+static int launch_factor(const Geom& G, T* A, T* Tws, int level, int p, int64_t nodes,
+                         cudaStream_t s) {
+    if (nodes <= 0) return 0;
+    const int wp = std::min<int>(kPW, G.ncols - 32 * p);
+    const int rgmax = level < 0 ? (int)std::min<int64_t>(G.b, G.mrows) : 2 * wp + 32 * p;
+    const size_t smem = panel_factor_smem<T>(wp, rgmax);
+    cudaError_t e = allow_smem(panel_factor_kernel<T>, smem);
+    if (e == cudaSuccess) {
+        panel_factor_kernel<T><<<dim3((unsigned)nodes), kThreads, smem, s>>>(G, A, Tws, level, p);
+        e = cudaGetLastError();
+    }
+    if (e != cudaSuccess) {
+        g_last_cuda_error = (int)e;
+        return CAQR_ERR_CUDA;
+    }
+    return 0;
+}
+
+template <typename T>
+static int launch_update(const Geom& G, const T* A, const T* Tws, int level, int p, int64_t nodes,
+                         T* C, int64_t ldc, int64_t cfirst, int64_t ccount, int trans,
+                         cudaStream_t s) {
+    if (nodes <= 0 || ccount <= 0) return 0;
+    const int wp = std::min<int>(kPW, G.ncols - 32 * p);
+    const int rgmax = level < 0 ? (int)std::min<int64_t>(G.b, G.mrows) : 2 * wp + 32 * p;
+    const size_t smem = panel_update_smem<T>(rgmax);
+    cudaError_t e = allow_smem(panel_update_kernel<T>, smem);
+    if (e == cudaSuccess) {
+        dim3 grid((unsigned)nodes, (unsigned)ceil_div(ccount, 32));
+        panel_update_kernel<T><<<grid, kThreads, smem, s>>>(G, A, Tws, level, p, C, ldc, cfirst,
+                                                            ccount, trans);
+        e = cudaGetLastError();
+    }
+    if (e != cudaSuccess) {
+        g_last_cuda_error = (int)e;
+        return CAQR_ERR_CUDA;
+    }
+    return 0;
+}
+
+// TSQR of one panel group (Fig. 4 minus the trailing update): every leaf's
+// panels (factor + intra-group trailing update), then every tree level.
+template <typename T>
+static int factor_group(const Geom& G, T* A, T* Tws, bool do_leaves, cudaStream_t s) {
+    int rc = 0;
+    if (do_leaves) {
+        for (int p = 0; p < G.npan && !rc; ++p) {
+            rc = launch_factor<T>(G, A, Tws, -1, p, G.L, s);
+            if (!rc && p + 1 < G.npan)
+                rc = launch_update<T>(G, A, Tws, -1, p, G.L, A, G.lda, G.col0 + 32 * (p + 1),
+                                      G.ncols - 32 * (p + 1), 1, s);
+        }
+    }
+    const int nl = tree_levels(G.L);
+    for (int lv = 0; lv < nl && !rc; ++lv) {
+        const int64_t nm = merges_at(G.L, lv);
+        for (int p = 0; p < G.npan && !rc; ++p) {
+            rc = launch_factor<T>(G, A, Tws, lv, p, nm, s);
+            if (!rc && p + 1 < G.npan)
+                rc = launch_update<T>(G, A, Tws, lv, p, nm, A, G.lda, G.col0 + 32 * (p + 1),
+                                      G.ncols - 32 * (p + 1), 1, s);
+        }
+    }
+    return rc;
+}
+
+// C[rows of the group, cfirst:cfirst+ccount] <- Q_g^T C (trans) or Q_g C.
+// Q_g^T = (tree top)^T ... (tree level 0)^T (leaves)^T, each node's panels in
+// order 0..npan-1; Q_g is the reverse.
+template <typename T>
+static int apply_group(const Geom& G, const T* A, const T* Tws, bool do_leaves, T* C,
+                       int64_t ldc, int64_t cfirst, int64_t ccount, int trans, cudaStream_t s) {
+    int rc = 0;
+    const int nl = tree_levels(G.L);
+    if (trans) {
+        if (do_leaves)
+            for (int p = 0; p < G.npan && !rc; ++p)
+                rc = launch_update<T>(G, A, Tws, -1, p, G.L, C, ldc, cfirst, ccount, 1, s);
+        for (int lv = 0; lv < nl && !rc; ++lv)
+            for (int p = 0; p < G.npan && !rc; ++p)
+                rc = launch_update<T>(G, A, Tws, lv, p, merges_at(G.L, lv), C, ldc, cfirst, ccount,
+                                      1, s);
+    } else {
+        for (int lv = nl - 1; lv >= 0 && !rc; --lv)
+            for (int p = G.npan - 1; p >= 0 && !rc; --p)
+                rc = launch_update<T>(G, A, Tws, lv, p, merges_at(G.L, lv), C, ldc, cfirst, ccount,
+                                      0, s);
+        if (do_leaves)
+            for (int p = G.npan - 1; p >= 0 && !rc; --p)
+                rc = launch_update<T>(G, A, Tws, -1, p, G.L, C, ldc, cfirst, ccount, 0, s);
+    }
+    return rc;
+}
+
+template <typename T>
+static int launch_extract_r(int64_t n, const T* A, int64_t lda, T* R, int64_t ldr, cudaStream_t s) {
+    if (n <= 0) return 0;
+    dim3 grid((unsigned)std::min<int64_t>(ceil_div(n, 256), 64), (unsigned)n);
+    extract_r_kernel<T><<<grid, 256, 0, s>>>(n, A, lda, R, ldr);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) {
+        g_last_cuda_error = (int)e;
+        return CAQR_ERR_CUDA;
+    }
+    return 0;
+}
+
+// ---- the ABI bodies ---------------------------------------------------------
+template <typename T>
+static int factor_impl(int64_t m, int64_t n, T* A, int64_t lda, T* R, int64_t ldr, void* ws,
+                       size_t ws_bytes, const caqr_opts* opts, cudaStream_t s, int dtype) {
+    if (m < 0) return -1;
+    if (n < 0 || n > m) return -2;
+    if (!A) return -3;
+    if (lda < std::max<int64_t>(1, m)) return -4;
+    if (!R) return -5;
+    if (ldr < std::max<int64_t>(1, n)) return -6;
+    Plan pl;
+    int rc = make_plan(m, n, dtype, opts, 9, &pl);
+    if (rc) return rc;
+    if (m == 0 || n == 0) return 0;
+    if (!ws) return -7;
+    if (ws_bytes < plan_ws_bytes(pl)) return -8;
+    T* Tws = static_cast<T*>(ws);
+    for (int64_t g = 0; g < pl.ngroups && !rc; ++g) {
+        const Geom G = group_geom(pl, g, lda);
+        rc = factor_group<T>(G, A, Tws, true, s);
+        const int64_t trail0 = G.col0 + G.ncols;
+        if (!rc && trail0 < n)  // CAQR trailing update
+            rc = apply_group<T>(G, A, Tws, true, A, lda, trail0, n - trail0, 1, s);
+        Tws += group_t_elems(G);
+    }
+    if (!rc) rc = launch_extract_r<T>(n, A, lda, R, ldr, s);
+    return rc;
+}
+
+template <typename T>
+static int apply_impl(int64_t m, int64_t n, const T* A, int64_t lda, const void* ws, int64_t k,
+                      T* C, int64_t ldc, const caqr_opts* opts, cudaStream_t s, int dtype,
+                      int trans) {
+    if (m < 0) return -1;
+    if (n < 0 || n > m) return -2;
+    if (!A) return -3;
+    if (lda < std::max<int64_t>(1, m)) return -4;
+    if (k < 0) return -6;
+    if (!C) return -7;
+    if (ldc < std::max<int64_t>(1, m)) return -8;
+    Plan pl;
+    int rc = make_plan(m, n, dtype, opts, 9, &pl);
+    if (rc) return rc;
+    if (m == 0 || n == 0 || k == 0) return 0;
+    if (!ws) return -5;
+    const T* base = static_cast<const T*>(ws);
+    // group offsets into the workspace
+    const T* tws[1024];
+    int64_t ng = pl.ngroups;
+    if (ng > 1024) return CAQR_ERR_UNSUPPORTED;
+    {
+        const T* t = base;
+        for (int64_t g = 0; g < ng; ++g) {
+            tws[g] = t;
+            t += group_t_elems(group_geom(pl, g, lda));
+        }
+    }
+    if (trans) {
+        for (int64_t g = 0; g < ng && !rc; ++g)
+            rc = apply_group<T>(group_geom(pl, g, lda), A, tws[g], true, C, ldc, 0, k, 1, s);
+    } else {
+        for (int64_t g = ng - 1; g >= 0 && !rc; --g)
+            rc = apply_group<T>(group_geom(pl, g, lda), A, tws[g], true, C, ldc, 0, k, 0, s);
+    }
+    return rc;
+}
+
+template <typename T>
+static int form_q_impl(int64_t m, int64_t n, const T* A, int64_t lda, const void* ws, T* Q,
+                       int64_t ldq, const caqr_opts* opts, cudaStream_t s, int dtype) {
+    if (m < 0) return -1;
+    if (n < 0 || n > m) return -2;
+    if (!A) return -3;
+    if (lda < std::max<int64_t>(1, m)) return -4;
+    if (!Q) return -6;
+    if (ldq < std::max<int64_t>(1, m)) return -7;
+    if (m == 0 || n == 0) return 0;
+    if (!ws) return -5;
+    dim3 grid((unsigned)std::min<int64_t>(ceil_div(m, 256), 1024), (unsigned)n);
+    set_identity_kernel<T><<<grid, 256, 0, s>>>(m, n, Q, ldq);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) {
+        g_last_cuda_error = (int)e;
+        return CAQR_ERR_CUDA;
+    }
+    const int rc = apply_impl<T>(m, n, A, lda, ws, n, Q, ldq, opts, s, dtype, 0);
+    return rc == -6 ? -7 : rc;
+}
+
+// Combine geometry: P slots of n rows (the leaves are the given R factors).
+static Geom combine_geom(int P, int64_t n, int64_t ld) {
+    Geom G;
+    G.lda = ld;
+    G.row0 = 0;
+    G.col0 = 0;
+    G.mrows = (int64_t)P * n;
+    G.ncols = (int32_t)n;
+    G.npan = (int32_t)ceil_div(n, kPW);
+    G.b = n;
+    G.L = P;
+    return G;
+}
+
+template <typename T>
+static int combine_impl(int P, int64_t n, T* Rs, int64_t ld, T* R, int64_t ldr, void* ws,
+                        size_t ws_bytes, cudaStream_t s, int dtype) {
+    if (P < 1) return -1;
+    if (n < 0 || n > kMaxGroup) return -2;
+    if (!Rs) return -3;
+    if (ld < std::max<int64_t>(1, (int64_t)P * n)) return -4;
+    if (!R) return -5;
+    if (ldr < std::max<int64_t>(1, n)) return -6;
+    if (n == 0) return 0;
+    if (!ws) return -7;
+    if (ws_bytes < caqr_combine_workspace_bytes(P, n, dtype)) return -8;
+    const Geom G = combine_geom(P, n, ld);
+    int rc = factor_group<T>(G, Rs, static_cast<T*>(ws), false, s);
+    if (!rc) rc = launch_extract_r<T>(n, Rs, ld, R, ldr, s);
+    return rc;
+}
+
+template <typename T>
+static int combine_apply_impl(int P, int64_t n, const T* Rs, int64_t ld, const void* ws, int trans,
+                              int64_t k, T* C, int64_t ldc, cudaStream_t s) {
+    if (P < 1) return -1;
+    if (n < 0 || n > kMaxGroup) return -2;
+    if (!Rs) return -3;
+    if (ld < std::max<int64_t>(1, (int64_t)P * n)) return -4;
+    if (k < 0) return -7;
+    if (!C) return -8;
+    if (ldc < std::max<int64_t>(1, (int64_t)P * n)) return -9;
+    if (n == 0 || k == 0) return 0;
+    if (!ws) return -5;
+    const Geom G = combine_geom(P, n, ld);
+    return apply_group<T>(G, Rs, static_cast<const T*>(ws), false, C, ldc, 0, k, trans ? 1 : 0, s);
+}
+
+}  // namespace caqr
+
+using namespace caqr;
+
+extern "C" {
+
+size_t caqr_workspace_bytes(int64_t m, int64_t n, int dtype, const caqr_opts* opts) {
+    if (m < 0 || n < 0 || n > m || (dtype != CAQR_F32 && dtype != CAQR_F64)) return 0;
+    Plan pl;
+    if (make_plan(m, n, dtype, opts, 4, &pl)) return 0;
+    return std::max<size_t>(plan_ws_bytes(pl), 256);
+}
+
+int caqr_factor_f32(int64_t m, int64_t n, float* A, int64_t lda, float* R, int64_t ldr, void* ws,
+                    size_t ws_bytes, const caqr_opts* opts, caqr_stream_t stream) {
+    return factor_impl<float>(m, n, A, lda, R, ldr, ws, ws_bytes, opts, stream, CAQR_F32);
+}
+int caqr_factor_f64(int64_t m, int64_t n, double* A, int64_t lda, double* R, int64_t ldr,
+                    void* ws, size_t ws_bytes, const caqr_opts* opts, caqr_stream_t stream) {
+    return factor_impl<double>(m, n, A, lda, R, ldr, ws, ws_bytes, opts, stream, CAQR_F64);
+}
+int caqr_apply_qt_f32(int64_t m, int64_t n, const float* A, int64_t lda, const void* ws, int64_t k,
+                      float* C, int64_t ldc, const caqr_opts* opts, caqr_stream_t stream) {
+    return apply_impl<float>(m, n, A, lda, ws, k, C, ldc, opts, stream, CAQR_F32, 1);
+}
+int caqr_apply_qt_f64(int64_t m, int64_t n, const double* A, int64_t lda, const void* ws,
+                      int64_t k, double* C, int64_t ldc, const caqr_opts* opts,
+                      caqr_stream_t stream) {
+    return apply_impl<double>(m, n, A, lda, ws, k, C, ldc, opts, stream, CAQR_F64, 1);
+}
+int caqr_apply_q_f32(int64_t m, int64_t n, const float* A, int64_t lda, const void* ws, int64_t k,
+                     float* C, int64_t ldc, const caqr_opts* opts, caqr_stream_t stream) {
+    return apply_impl<float>(m, n, A, lda, ws, k, C, ldc, opts, stream, CAQR_F32, 0);
+}
+int caqr_apply_q_f64(int64_t m, int64_t n, const double* A, int64_t lda, const void* ws, int64_t k,
+                     double* C, int64_t ldc, const caqr_opts* opts, caqr_stream_t stream) {
+    return apply_impl<double>(m, n, A, lda, ws, k, C, ldc, opts, stream, CAQR_F64, 0);
+}
+int caqr_form_q_f32(int64_t m, int64_t n, const float* A, int64_t lda, const void* ws, float* Q,
+                    int64_t ldq, const caqr_opts* opts, caqr_stream_t stream) {
+    return form_q_impl<float>(m, n, A, lda, ws, Q, ldq, opts, stream, CAQR_F32);
+}
+int caqr_form_q_f64(int64_t m, int64_t n, const double* A, int64_t lda, const void* ws, double* Q,
+                    int64_t ldq, const caqr_opts* opts, caqr_stream_t stream) {
+    return form_q_impl<double>(m, n, A, lda, ws, Q, ldq, opts, stream, CAQR_F64);
+}
+
+size_t caqr_combine_workspace_bytes(int P, int64_t n, int dtype) {
+    if (P < 1 || n < 0 || n > kMaxGroup || (dtype != CAQR_F32 && dtype != CAQR_F64)) return 0;
+    if (n == 0) return 256;
+    const Geom G = combine_geom(P, n, (int64_t)P * n);
+    // T blocks + room for P contiguous n x n blocks (the NCCL receive buffer of
+    // caqr_dist_factor_*).
+    const size_t elems = group_t_elems(G) + (size_t)P * n * n;
+    return elems * (dtype == CAQR_F64 ? 8 : 4);
+}
+int caqr_combine_f32(int P, int64_t n, float* Rs, int64_t ld, float* R, int64_t ldr, void* ws,
+                     size_t ws_bytes, caqr_stream_t stream) {
+    return combine_impl<float>(P, n, Rs, ld, R, ldr, ws, ws_bytes, stream, CAQR_F32);
+}
+int caqr_combine_f64(int P, int64_t n, double* Rs, int64_t ld, double* R, int64_t ldr, void* ws,
+                     size_t ws_bytes, caqr_stream_t stream) {
+    return combine_impl<double>(P, n, Rs, ld, R, ldr, ws, ws_bytes, stream, CAQR_F64);
+}
+int caqr_combine_apply_f32(int P, int64_t n, const float* Rs, int64_t ld, const void* ws, int trans,
+                           int64_t k, float* C, int64_t ldc, caqr_stream_t stream) {
+    return combine_apply_impl<float>(P, n, Rs, ld, ws, trans, k, C, ldc, stream);
+}
+int caqr_combine_apply_f64(int P, int64_t n, const double* Rs, int64_t ld, const void* ws,
+                           int trans, int64_t k, double* C, int64_t ldc, caqr_stream_t stream) {
+    return combine_apply_impl<double>(P, n, Rs, ld, ws, trans, k, C, ldc, stream);
+}
+
+const char* caqr_strerror(int info) {
+    if (info == 0) return "success";
+    if (info == CAQR_ERR_CUDA) return "CUDA launch failed (see caqr_last_cuda_error)";
+    if (info == CAQR_ERR_NCCL) return "NCCL call failed";
+    if (info == CAQR_ERR_UNSUPPORTED) return "unsupported size";
+    if (info < 0) return "illegal argument (-info = position)";
+    return "unknown";
+}
+int caqr_last_cuda_error(void) { return g_last_cuda_error; }
+const char* caqr_build_info(void) {
+    return "libcaqr: sm_100a TSQR/CAQR (panel_factor + panel_update kernels, FFMA/DFMA), "
+           "built " __DATE__ " " __TIME__;
+}
+
+int caqr_plan_info(int64_t m, int64_t n, int dtype, const caqr_opts* opts, int64_t out[8]) {
+    if (!out) return -5;
+    if (m < 0) return -1;
+    if (n < 0 || n > m) return -2;
+    if (dtype != CAQR_F32 && dtype != CAQR_F64) return -3;
+    Plan pl;
+    int rc = make_plan(m, n, dtype, opts, 4, &pl);
+    if (rc) return rc;
+    std::memset(out, 0, 8 * sizeof(int64_t));
+    out[0] = pl.b;
+    out[1] = pl.nb;
+    out[2] = pl.ngroups;
+    if (pl.ngroups == 0) return 0;
+    const Geom G = group_geom(pl, 0, m);
+    out[3] = G.L;
+    out[4] = tree_levels(G.L);
+    out[5] = G.npan;
+    int64_t launches = 1;  // extract_r
+    for (int64_t g = 0; g < pl.ngroups; ++g) {
+        const Geom Gg = group_geom(pl, g, m);
+        const int nl = tree_levels(Gg.L);
+        launches += (int64_t)(nl + 1) * (2 * Gg.npan - 1);
+        if (Gg.col0 + Gg.ncols < n) launches += (int64_t)(nl + 1) * Gg.npan;
+    }
+    out[6] = launches;
+    return 0;
+}
+
+}  // extern "C"

@@ -1,0 +1,457 @@
+// tsqr_kernels.cuh -- sm_100a device code of the TSQR / CAQR hot path.
+//
+// Two kernels carry the whole method:
+//
+//  panel_factor_kernel   Householder QR of one <=32-column panel of one tree
+//                        node (a leaf row block -- the paper's "factor",
+//                        or a stacked pair of R factors -- its
+//                        "factor_tree"), entirely in shared memory,
+//                        one CTA per node.  Per column: warp-shuffle norm,
+//                        reflector, warp-shuffle dot products s = A^T v and the
+//                        rank-1 update A -= tau v s^T (Fig. 5), then
+//                        the compact-WY factor T from the inner products of the
+//                        vectors.
+//  panel_update_kernel   C <- (I - V T V^T)^T C (or without ^T) for one node and
+//                        one 32-column block of C: W = V^T C, W = T^T W,
+//                        C -= V W -- the blocked trailing update
+//                        used horizontally across leaves ("apply_qt_h",
+//                        P:L665-668) and on the gathered rows of tree nodes
+//                        ("apply_qt_tree", Fig. 3(c,d)).
+//
+// A tree node's rows are "gathered": a leaf is one contiguous row segment; a
+// merge of R_a and R_b (binary tree) is the segment holding R_a's
+// rows of the current panel followed by the segment holding R_b's top rows.
+// Masks keep the stacked-triangle structure ("possibly exploiting
+// the sparsity pattern") and keep the leaves' vectors that share those rows
+// untouched (tree vectors overwrite exactly the R slots).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace caqr {
+
+constexpr int kPW = 32;        // max reflectors per panel step (panel width)
+constexpr int kThreads = 256;  // 8 warps
+constexpr int kWarps = kThreads / 32;
+constexpr int kTS = 33;        // stride of 32x32 scratch tiles in shared memory
+
+// Geometry of one TSQR panel group (a column panel of width ncols <= 256 that
+// starts at row0 = col0 of A; the grid redrawn "nb rows lower").
+struct Geom {
+    int64_t lda;
+    int64_t row0;   // first row of the group
+    int64_t mrows;  // rows of the group (m - row0)
+    int64_t col0;   // first column of the group
+    int64_t b;      // leaf height
+    int64_t L;      // number of leaves
+    int32_t ncols;  // group width
+    int32_t npan;   // ceil(ncols / 32)
+};
+
+// The gathered rows of node `node` at tree `level` (-1 = leaves) for panel p.
+struct NodeRows {
+    int64_t r0, r1;  // first absolute row of segment 0 / segment 1
+    int32_t n0, n1;  // rows in segment 0 / 1
+    int32_t merge;   // 0 = leaf, 1 = merge of two R factors
+    int64_t tblk;    // index of this (node, panel)'s 32x32 T block in the workspace
+};
+
+__device__ __forceinline__ NodeRows node_rows(const Geom& g, int level, int64_t node, int p,
+                                              int wp) {
+    NodeRows nr;
+    if (level < 0) {
+        const int64_t s = g.row0 + node * g.b;
+        const int64_t h = min(g.b, g.mrows - node * g.b);
+        nr.r0 = s + 32 * p;
+        nr.n0 = (int32_t)(h - 32 * p > 0 ? h - 32 * p : 0);
+        nr.r1 = 0;
+        nr.n1 = 0;
+        nr.merge = 0;
+        nr.tblk = node * g.npan + p;
+    } else {
+        const int64_t a = node << (level + 1);
+        const int64_t bb = a + (int64_t(1) << level);
+        const int64_t hb = min(g.b, g.mrows - bb * g.b);
+        nr.r0 = g.row0 + a * g.b + 32 * p;
+        nr.n0 = wp;
+        nr.r1 = g.row0 + bb * g.b;
+        nr.n1 = (int32_t)(32 * p + wp < hb ? 32 * p + wp : hb);
+        nr.merge = 1;
+        nr.tblk = (g.L + bb) * g.npan + p;
+    }
+    return nr;
+}
+
+// Absolute row of gathered row r.
+__device__ __forceinline__ int64_t gathered_row(const NodeRows& nr, int r) {
+    return r < nr.n0 ? nr.r0 + r : nr.r1 + (r - nr.n0);
+}
+
+// Is entry (gathered row r, panel column jj) of the panel stored in A for this
+// node?  Leaves: every entry (R on/above the diagonal, v below).  Merges: R_a's
+// rows hold R on and above the diagonal only (below it sit leaf vectors);
+// R_b's rows hold an upper-triangular R (factor input) / V_2 (tree vectors)
+// only -- local row i <= 32p + jj.
+__device__ __forceinline__ bool panel_entry_stored(const NodeRows& nr, int r, int jj, int p) {
+    if (!nr.merge) return true;
+    if (r < nr.n0) return r <= jj;
+    return (r - nr.n0) <= 32 * p + jj;
+}
+
+template <typename T>
+__device__ __forceinline__ T warp_sum(T v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+
+// Column stride (elements) of a column-major shared tile with >= rows rows:
+// rows rounded up to 32, plus 16 bytes, so that 16-byte vector loads by lanes
+// reading 8 different columns at the same rows hit 8 disjoint bank groups.
+template <typename T>
+__host__ __device__ __forceinline__ int smem_col_stride(int rows) {
+    const int r32 = (rows + 31) & ~31;
+    return r32 + int(16 / sizeof(T));
+}
+
+// ---------------------------------------------------------------------------
+// Reflector of panel column j (xLARFG, reading S1), computed by ONE
+// warp: alpha = P[j][j], sigma = sum_{r>j} P[r][j]^2 (warp-shuffle reduction),
+// beta = -copysign(sqrt(alpha^2+sigma), alpha), tau = (beta-alpha)/beta,
+// v = P[j+1:, j] / (alpha - beta); P[j][j] <- beta.  sigma == 0 -> tau = 0.
+// ---------------------------------------------------------------------------
+template <typename T>
+__device__ __forceinline__ void make_reflector(T* P, int RGP, int RG, int j, T* tau_s, int lane) {
+    T* col = P + (size_t)j * RGP;
+    const T alpha = (j < RG) ? col[j] : T(0);
+    T sigma = T(0);
+    for (int r = j + 1 + lane; r < RG; r += 32) {
+        const T x = col[r];
+        sigma = fma(x, x, sigma);
+    }
+    sigma = warp_sum(sigma);
+    T tau = T(0);
+    if (j < RG && sigma != T(0)) {
+        const T mu = sqrt(fma(alpha, alpha, sigma));
+        const T beta = -copysign(mu, alpha);
+        tau = (beta - alpha) / beta;
+        const T scale = T(1) / (alpha - beta);
+        for (int r = j + 1 + lane; r < RG; r += 32) col[r] *= scale;
+        __syncwarp();
+        if (lane == 0) col[j] = beta;
+    }
+    if (lane == 0) tau_s[j] = tau;
+    __syncwarp();
+}
+
+// ---------------------------------------------------------------------------
+// panel_factor_kernel: grid = nodes of this level, block = 256 threads.
+// Shared: P (wp columns x RGP), G (32x33), Tm (32x33), tau (32).
+// ---------------------------------------------------------------------------
+template <typename T>
+__global__ void __launch_bounds__(kThreads)
+panel_factor_kernel(Geom g, T* A, T* __restrict__ Tws, int level, int p) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int wp = min(kPW, g.ncols - 32 * p);
+    const NodeRows nr = node_rows(g, level, blockIdx.x, p, wp);
+    const int RG = nr.n0 + nr.n1;
+    const int RGP = smem_col_stride<T>(RG);
+    T* P = reinterpret_cast<T*>(smem_raw);
+    T* G = P + (size_t)wp * RGP;
+    T* Tm = G + kPW * kTS;
+    T* tau_s = Tm + kPW * kTS;
+    const int64_t c0 = g.col0 + 32 * p;
+
+    // ---- stage: coalesced column loads (lanes along rows) with structure masks
+    for (int jj = warp; jj < wp; jj += kWarps) {
+        const T* col = A + (c0 + jj) * g.lda;
+        T* pc = P + (size_t)jj * RGP;
+        for (int r = lane; r < RG; r += 32)
+            pc[r] = panel_entry_stored(nr, r, jj, p) ? col[gathered_row(nr, r)] : T(0);
+    }
+    __syncthreads();
+
+    // ---- unblocked Householder over the panel columns ----------
+    // Column c is owned by warp c % 8.  After reflector j is published, each
+    // warp applies it to its columns c > j (dot via shuffles, rank-1 update);
+    // the owner of column j+1 builds reflector j+1 right after updating it, so
+    // one CTA barrier per column suffices.
+    if (warp == 0) make_reflector(P, RGP, RG, 0, tau_s, lane);
+    __syncthreads();
+    for (int j = 0; j < wp; ++j) {
+        const T tau = tau_s[j];
+        const T* v = P + (size_t)j * RGP;
+        int c = j + 1 + ((warp - (j + 1)) % kWarps + kWarps) % kWarps;  // first owned c > j
+        for (; c < wp; c += kWarps) {
+            T* a = P + (size_t)c * RGP;
+            if (tau != T(0)) {
+                T s = T(0);
+                for (int r = j + 1 + lane; r < RG; r += 32) s = fma(v[r], a[r], s);
+                s = warp_sum(s);
+                s = (s + a[j]) * tau;
+                __syncwarp();
+                for (int r = j + 1 + lane; r < RG; r += 32) a[r] = fma(-s, v[r], a[r]);
+                if (lane == 0) a[j] -= s;
+                __syncwarp();
+            }
+            if (c == j + 1) make_reflector(P, RGP, RG, c, tau_s, lane);
+        }
+        __syncthreads();
+    }
+
+    // ---- compact-WY T (LAPACK xLARFT, forward/columnwise) -------
+    // G[i][j] = v_i . v_j (i < j) with unit heads; T[j][j] = tau_j,
+    // T[0:j, j] = -tau_j T[0:j, 0:j] G[0:j, j].
+    for (int j = warp; j < wp; j += kWarps) {
+        const T* vj = P + (size_t)j * RGP;
+        for (int i = 0; i < j; ++i) {
+            const T* vi = P + (size_t)i * RGP;
+            T s = T(0);
+            for (int r = j + 1 + lane; r < RG; r += 32) s = fma(vi[r], vj[r], s);
+            s = warp_sum(s);
+            if (lane == 0) G[i * kTS + j] = s + (j < RG ? vi[j] : T(0));
+        }
+    }
+    __syncthreads();
+    if (warp == 0 && lane < wp) {
+        const int i = lane;
+        Tm[i * kTS + i] = tau_s[i];
+        for (int j = i + 1; j < wp; ++j) {
+            T t = T(0);
+            for (int k = i; k < j; ++k) t = fma(Tm[i * kTS + k], G[k * kTS + j], t);
+            Tm[i * kTS + j] = -tau_s[j] * t;
+        }
+    }
+    __syncthreads();
+
+    // ---- write back: panel (masked) to A, T (32x32 column-major) to ws ------
+    for (int jj = warp; jj < wp; jj += kWarps) {
+        T* col = A + (c0 + jj) * g.lda;
+        const T* pc = P + (size_t)jj * RGP;
+        for (int r = lane; r < RG; r += 32)
+            if (panel_entry_stored(nr, r, jj, p)) col[gathered_row(nr, r)] = pc[r];
+    }
+    T* tb = Tws + nr.tblk * (kPW * kPW);
+    for (int e = threadIdx.x; e < kPW * kPW; e += kThreads) {
+        const int r = e & 31, c = e >> 5;
+        tb[e] = (r <= c && c < wp) ? Tm[r * kTS + c] : T(0);
+    }
+}
+
+template <typename T>
+inline size_t panel_factor_smem(int wp, int RGmax) {
+    return sizeof(T) * ((size_t)wp * smem_col_stride<T>(RGmax) + 2 * kPW * kTS + kPW);
+}
+
+// ---------------------------------------------------------------------------
+// panel_update_kernel: C[gathered rows, block] <- op(I - V T V^T) C.
+// grid.x = nodes, grid.y = 32-column blocks of C's [cfirst, cfirst+ccount).
+// trans = 1: Q^T (W = T^T V^T C), trans = 0: Q (W = T V^T C).
+// Shared: Vs, Cs (32 columns x RGP, column-major, rows zero-padded to 32),
+// Wp (4 K-split partials of 32x33), Tt (32x33), W (32x33).
+// ---------------------------------------------------------------------------
+template <typename T>
+struct Vec4;  // 16-byte vector of T
+template <>
+struct Vec4<float> {
+    using type = float4;
+    static constexpr int n = 4;
+};
+template <>
+struct Vec4<double> {
+    using type = double2;
+    static constexpr int n = 2;
+};
+
+template <typename T>
+__device__ __forceinline__ T vget(const float4& v, int i) {
+    return i == 0 ? v.x : i == 1 ? v.y : i == 2 ? v.z : v.w;
+}
+template <typename T>
+__device__ __forceinline__ T vget(const double2& v, int i) {
+    return i == 0 ? v.x : v.y;
+}
+
+template <typename T>
+__global__ void __launch_bounds__(kThreads)
+panel_update_kernel(Geom g, const T* A, const T* __restrict__ Tws, int level, int p, T* C,
+                    int64_t ldc, int64_t cfirst, int64_t ccount, int trans) {
+    using V4 = typename Vec4<T>::type;
+    constexpr int VN = Vec4<T>::n;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int wp = min(kPW, g.ncols - 32 * p);
+    const NodeRows nr = node_rows(g, level, blockIdx.x, p, wp);
+    const int RG = nr.n0 + nr.n1;
+    if (RG == 0) return;
+    const int R32 = (RG + 31) & ~31;
+    const int RGP = smem_col_stride<T>(RG);
+    const int64_t cb0 = cfirst + 32 * (int64_t)blockIdx.y;
+    const int ncb = (int)(cfirst + ccount - cb0 < 32 ? cfirst + ccount - cb0 : 32);
+    T* Vs = reinterpret_cast<T*>(smem_raw);
+    T* Cs = Vs + 32 * (size_t)RGP;
+    T* Wp = Cs + 32 * (size_t)RGP;  // 4 x 32 x kTS
+    T* Tt = Wp + 4 * 32 * kTS;
+    T* W = Tt + 32 * kTS;
+    const int64_t c0 = g.col0 + 32 * p;
+
+    // ---- stage V (implicit unit heads, structure masks) and C ---------------
+    for (int jj = warp; jj < 32; jj += kWarps) {
+        T* vs = Vs + (size_t)jj * RGP;
+        T* cs = Cs + (size_t)jj * RGP;
+        const T* acol = A + (c0 + jj) * g.lda;
+        const T* ccol = C + (cb0 + jj) * ldc;
+        for (int r = lane; r < R32; r += 32) {
+            T v = T(0), cv = T(0);
+            if (r < RG) {
+                if (jj < wp) {
+                    if (!nr.merge) {
+                        v = r > jj ? acol[gathered_row(nr, r)] : (r == jj ? T(1) : T(0));
+                    } else if (r < nr.n0) {
+                        v = (r == jj) ? T(1) : T(0);
+                    } else {
+                        v = (r - nr.n0) <= 32 * p + jj ? acol[nr.r1 + (r - nr.n0)] : T(0);
+                    }
+                }
+                if (jj < ncb) cv = ccol[gathered_row(nr, r)];
+            }
+            vs[r] = v;
+            cs[r] = cv;
+        }
+    }
+    {
+        const T* tb = Tws + nr.tblk * (kPW * kPW);
+        for (int e = tid; e < kPW * kPW; e += kThreads) Tt[(e & 31) * kTS + (e >> 5)] = tb[e];
+    }
+    __syncthreads();
+
+    // ---- W = V^T C : 4-way split over rows x 2 column halves per warp -------
+    {
+        const int ks = warp & 3, ch = warp >> 2;
+        const int jg = lane & 7, cg = lane >> 3;  // jj = jg + 8e (e<4), c = 16ch + cg + 4e (e<4)
+        const int chunk = R32 / 4;                // multiple of 8
+        const int rbeg = ks * chunk, rend = rbeg + chunk;
+        T acc[4][4];
+#pragma unroll
+        for (int a = 0; a < 4; ++a)
+#pragma unroll
+            for (int b2 = 0; b2 < 4; ++b2) acc[a][b2] = T(0);
+        for (int r = rbeg; r < rend; r += VN) {
+            V4 vv[4], cc[4];
+#pragma unroll
+            for (int e = 0; e < 4; ++e)
+                vv[e] = *reinterpret_cast<const V4*>(Vs + (size_t)(jg + 8 * e) * RGP + r);
+#pragma unroll
+            for (int e = 0; e < 4; ++e)
+                cc[e] = *reinterpret_cast<const V4*>(Cs + (size_t)(16 * ch + cg + 4 * e) * RGP + r);
+#pragma unroll
+            for (int q = 0; q < VN; ++q)
+#pragma unroll
+                for (int a = 0; a < 4; ++a)
+#pragma unroll
+                    for (int b2 = 0; b2 < 4; ++b2)
+                        acc[a][b2] = fma(vget<T>(vv[a], q), vget<T>(cc[b2], q), acc[a][b2]);
+        }
+#pragma unroll
+        for (int a = 0; a < 4; ++a)
+#pragma unroll
+            for (int b2 = 0; b2 < 4; ++b2)
+                Wp[(ks * 32 + jg + 8 * a) * kTS + 16 * ch + cg + 4 * b2] = acc[a][b2];
+    }
+    __syncthreads();
+    // reduce the 4 partials (fixed order: deterministic)
+    for (int e = tid; e < 32 * 32; e += kThreads) {
+        const int jj = e >> 5, c = e & 31;
+        T s = Wp[(0 * 32 + jj) * kTS + c];
+        s += Wp[(1 * 32 + jj) * kTS + c];
+        s += Wp[(2 * 32 + jj) * kTS + c];
+        s += Wp[(3 * 32 + jj) * kTS + c];
+        W[jj * kTS + c] = s;
+    }
+    __syncthreads();
+    // ---- W2 = T^T W (Q^T) or T W (Q); T upper triangular (Tt[r][c] = T[r][c])
+    T w2[4];
+    {
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            const int e = tid + q * kThreads;
+            const int jj = e >> 5, c = e & 31;
+            T s = T(0);
+            if (trans) {
+                for (int k = 0; k <= jj; ++k) s = fma(Tt[k * kTS + jj], W[k * kTS + c], s);
+            } else {
+                for (int k = jj; k < 32; ++k) s = fma(Tt[jj * kTS + k], W[k * kTS + c], s);
+            }
+            w2[q] = s;
+        }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+        const int e = tid + q * kThreads;
+        W[(e >> 5) * kTS + (e & 31)] = w2[q];
+    }
+    __syncthreads();
+
+    // ---- C -= V W2 : thread = (4 consecutive rows, 8 consecutive columns) ---
+    const int nq = R32 / 4;
+    for (int u = tid; u < nq * 4; u += kThreads) {
+        const int q = u % nq, cgrp = u / nq;
+        const int r = 4 * q, cbase = 8 * cgrp;
+        T acc[4][8];
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+#pragma unroll
+            for (int c = 0; c < 8; ++c) acc[i][c] = Cs[(size_t)(cbase + c) * RGP + r + i];
+        for (int jj = 0; jj < wp; ++jj) {
+            T vr[4];
+#pragma unroll
+            for (int h = 0; h < 4 / VN; ++h) {
+                const V4 t4 = *reinterpret_cast<const V4*>(Vs + (size_t)jj * RGP + r + h * VN);
+#pragma unroll
+                for (int q = 0; q < VN; ++q) vr[h * VN + q] = vget<T>(t4, q);
+            }
+#pragma unroll
+            for (int c = 0; c < 8; ++c) {
+                const T wv = W[jj * kTS + cbase + c];
+#pragma unroll
+                for (int i = 0; i < 4; ++i) acc[i][c] = fma(-vr[i], wv, acc[i][c]);
+            }
+        }
+#pragma unroll
+        for (int c = 0; c < 8; ++c) {
+            if (cbase + c >= ncb) break;
+            T* ccol = C + (cb0 + cbase + c) * ldc;
+#pragma unroll
+            for (int i = 0; i < 4; ++i)
+                if (r + i < RG) ccol[gathered_row(nr, r + i)] = acc[i][c];
+        }
+    }
+}
+
+template <typename T>
+inline size_t panel_update_smem(int RGmax) {
+    return sizeof(T) * (64 * (size_t)smem_col_stride<T>(RGmax) + 6 * 32 * kTS);
+}
+
+// R (n x n, ldr) <- triu(A[0:n, 0:n]).
+template <typename T>
+__global__ void extract_r_kernel(int64_t n, const T* __restrict__ A, int64_t lda,
+                                 T* __restrict__ R, int64_t ldr) {
+    const int64_t c = blockIdx.y;
+    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n;
+         r += (int64_t)gridDim.x * blockDim.x)
+        R[c * ldr + r] = r <= c ? A[c * lda + r] : T(0);
+}
+
+// Q (m x n, ldq) <- [I_n; 0].
+template <typename T>
+__global__ void set_identity_kernel(int64_t m, int64_t n, T* __restrict__ Q, int64_t ldq) {
+    const int64_t c = blockIdx.y;
+    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < m;
+         r += (int64_t)gridDim.x * blockDim.x)
+        Q[c * ldq + r] = r == c ? T(1) : T(0);
+}
+
+}  // namespace caqr

@@ -1,0 +1,83 @@
+"""C-ABI checks that need no GPU: the library builds, loads, exports every
+symbol include/caqr.h declares, and its host-side planner / argument checks
+behave as documented (LAPACK info codes, workspace sizes)."""
+import ctypes
+
+import pytest
+
+from paper_conf_ipps_andersonbdk11_b200 import build as cbuild
+from paper_conf_ipps_andersonbdk11_b200 import caqr
+
+
+@pytest.fixture(scope="module")
+def L():
+    cbuild.build()
+    return caqr.lib()
+
+
+def test_exports_every_header_symbol(L):
+    names = caqr.header_functions()
+    assert len(names) >= 20
+    missing = [n for n in names if not hasattr(L, n)]
+    assert not missing, missing
+
+
+def test_build_info(L):
+    assert b"sm_100a" in L.caqr_build_info()
+
+
+def test_sass_is_sm100a():
+    import subprocess
+
+    out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", caqr.LIB_PATH],
+                         capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+
+
+def test_workspace_bytes(L):
+    # one T block (32x32) per (leaf, panel) and per (merge, panel): 2*L*npan*1024 elems
+    assert caqr.caqr_workspace_bytes(4096, 16) == 2 * 16 * 1 * 1024 * 4
+    assert caqr.caqr_workspace_bytes(4096, 16, caqr.CAQR_F64) == 2 * 16 * 1 * 1024 * 8
+    assert caqr.caqr_workspace_bytes(1_000_000, 192) == 2 * 3907 * 6 * 1024 * 4
+    assert caqr.caqr_workspace_bytes(10, 11) == 0  # n > m
+    assert caqr.caqr_workspace_bytes(-1, 1) == 0
+    assert caqr.caqr_workspace_bytes(10, 2, 7) == 0  # bad dtype
+    assert caqr.caqr_workspace_bytes(100, 8, 0, caqr.make_opts(leaf_rows=100)) == 0  # not /32
+
+
+def test_plan_info(L):
+    p = caqr.caqr_plan_info(1_000_000, 192)
+    assert p["leaf_rows"] == 256 and p["panel_cols"] == 192 and p["groups"] == 1
+    assert p["leaves"] == 3907 and p["tree_levels"] == 12 and p["panels"] == 6
+    p = caqr.caqr_plan_info(8192, 8192)
+    assert p["panel_cols"] == 64 and p["groups"] == 128
+    p = caqr.caqr_plan_info(4096, 16, 0, caqr.make_opts(leaf_rows=128))
+    assert p["leaf_rows"] == 128 and p["leaves"] == 32 and p["tree_levels"] == 5
+
+
+def test_info_codes_without_gpu(L):
+    """Illegal arguments are rejected before any CUDA call (LAPACK info)."""
+    vp = ctypes.c_void_p
+    f = L.caqr_factor_f32
+    null = None
+    assert f(-1, 1, vp(8), 1, vp(8), 1, vp(8), 1 << 20, null, null) == -1
+    assert f(4, 5, vp(8), 4, vp(8), 5, vp(8), 1 << 20, null, null) == -2
+    assert f(4, 2, null, 4, vp(8), 2, vp(8), 1 << 20, null, null) == -3
+    assert f(4, 2, vp(8), 3, vp(8), 2, vp(8), 1 << 20, null, null) == -4
+    assert f(4, 2, vp(8), 4, null, 2, vp(8), 1 << 20, null, null) == -5
+    assert f(4, 2, vp(8), 4, vp(8), 1, vp(8), 1 << 20, null, null) == -6
+    assert f(4, 2, vp(8), 4, vp(8), 2, null, 1 << 20, null, null) == -7
+    assert f(4, 2, vp(8), 4, vp(8), 2, vp(8), 1, null, null) == -8
+    bad = caqr.Opts(100, 0)
+    assert f(4, 2, vp(8), 4, vp(8), 2, vp(8), 1 << 20, ctypes.byref(bad), null) == -9
+    # quick return
+    assert f(0, 0, vp(8), 1, vp(8), 1, null, 0, null, null) == 0
+    g = L.caqr_apply_qt_f32
+    assert g(4, 2, vp(8), 4, vp(8), -1, vp(8), 4, null, null) == -6
+    assert g(4, 2, vp(8), 4, vp(8), 3, vp(8), 2, null, null) == -8
+    h = L.caqr_form_q_f64
+    assert h(4, 2, vp(8), 4, vp(8), vp(8), 3, null, null) == -7
+    c = L.caqr_combine_f32
+    assert c(0, 4, vp(8), 4, vp(8), 4, vp(8), 1 << 20, null) == -1
+    assert c(2, 300, vp(8), 600, vp(8), 300, vp(8), 1 << 30, null) == -2
+    assert L.caqr_strerror(-3) and L.caqr_strerror(1)
