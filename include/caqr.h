@@ -184,6 +184,18 @@ int caqr_dist_factor_f64(caqr_dist *h, int64_t m_local, int64_t n, double *A, in
 const char *caqr_strerror(int info);
 int caqr_last_cuda_error(void);          /* cudaError_t of the last CAQR_ERR_CUDA (thread-local) */
 const char *caqr_build_info(void);       /* "sm_100a ..." */
+/* Launch tracing (profiling aid, not needed for correct use).
+ * caqr_trace_begin(cap): from now on every kernel the library launches (any
+ *   thread) is bracketed by two CUDA events recorded on its launching stream,
+ *   up to cap launches; 0, -1 (cap < 1), -2 (already tracing), CAQR_ERR_CUDA.
+ * caqr_trace_end(...): stops tracing, waits for the recorded events and fills
+ *   up to cap entries: kernel id (caqr_kernel_name), duration in ms, and the
+ *   host-computed algorithmic flops and bytes of that launch.  Returns the
+ *   number of launches recorded (may exceed cap).  Output pointers may be NULL. */
+int caqr_trace_begin(int capacity);
+int caqr_trace_end(int *kernel_ids, float *ms, double *flops, double *bytes, int cap);
+const char *caqr_kernel_name(int id);
+
 /* Plan introspection (host only; for tests and the bench's roofline bookkeeping).
  * Fills out[0..7] = {leaf_rows, panel_cols, groups, leaves(group 0),
  * tree_levels(group 0), panels(group 0), kernel_launches(factor), 0}.

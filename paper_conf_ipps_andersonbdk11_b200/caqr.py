@@ -84,6 +84,13 @@ def lib() -> ctypes.CDLL:
         L.caqr_build_info.restype = ctypes.c_char_p
         L.caqr_plan_info.argtypes = [i64, i64, ip, op, ctypes.POINTER(ctypes.c_int64)]
         L.caqr_plan_info.restype = ip
+        L.caqr_trace_begin.argtypes = [ip]
+        L.caqr_trace_begin.restype = ip
+        L.caqr_trace_end.argtypes = [ctypes.POINTER(ip), ctypes.POINTER(ctypes.c_float),
+                                     ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double), ip]
+        L.caqr_trace_end.restype = ip
+        L.caqr_kernel_name.argtypes = [ip]
+        L.caqr_kernel_name.restype = ctypes.c_char_p
         L.caqr_dist_unique_id.argtypes = [vp]
         L.caqr_dist_unique_id.restype = ip
         L.caqr_dist_create.argtypes = [ctypes.POINTER(vp), ip, ip, vp]
@@ -289,3 +296,21 @@ def qr_host(A_host, opts=None, stream=None, pinned_out=None):
     out = pinned_out if pinned_out is not None else torch.empty(R.shape, dtype=R.dtype, pin_memory=True)
     out.copy_(R, non_blocking=True)
     return out, A_dev, ws
+
+
+# ---- launch tracing (profiling aid) -----------------------------------------
+def caqr_trace_begin(capacity: int = 1 << 16) -> None:
+    _check("caqr_trace_begin", lib().caqr_trace_begin(capacity))
+
+
+def caqr_trace_end(capacity: int = 1 << 16):
+    """Stop tracing; return a list of (kernel_name, ms, flops, bytes), one per launch."""
+    L = lib()
+    ids = (ctypes.c_int * capacity)()
+    ms = (ctypes.c_float * capacity)()
+    fl = (ctypes.c_double * capacity)()
+    by = (ctypes.c_double * capacity)()
+    n = L.caqr_trace_end(ids, ms, fl, by, capacity)
+    n = min(n, capacity)
+    return [(L.caqr_kernel_name(ids[i]).decode(), float(ms[i]), float(fl[i]), float(by[i]))
+            for i in range(n)]

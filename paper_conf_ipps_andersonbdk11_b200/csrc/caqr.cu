@@ -8,15 +8,51 @@
 
 #include <algorithm>
 #include <cstdint>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 
 #include "../../include/caqr.h"
+#include "tsqr_fused.cuh"
 #include "tsqr_kernels.cuh"
 
 namespace caqr {
 
 static thread_local int g_last_cuda_error = 0;
+
+// ---- launch tracing (diagnostics: per-launch CUDA events on the launching
+// stream + host-computed algorithmic flops/bytes; see caqr_trace_begin) -------
+enum KernelId { K_PANEL_FACTOR = 0, K_PANEL_UPDATE = 1, K_EXTRACT_R = 2, K_SET_IDENTITY = 3,
+                K_TSQR_FUSED = 4, K_NUM = 5 };
+static const char* const kKernelNames[K_NUM] = {"panel_factor", "panel_update", "extract_r",
+                                                "set_identity", "tsqr_fused"};
+struct Trace {
+    std::mutex mu;
+    bool on = false;
+    int cap = 0, n = 0;
+    cudaEvent_t* ev = nullptr;
+    int* kid = nullptr;
+    double* flops = nullptr;
+    double* bytes = nullptr;
+};
+static Trace g_trace;
+struct TraceScope {  // records a start event now and a stop event at destruction
+    int slot = -1;
+    cudaStream_t s;
+    TraceScope(int k, double fl, double by, cudaStream_t st) : s(st) {
+        if (!g_trace.on) return;
+        std::lock_guard<std::mutex> lk(g_trace.mu);
+        if (!g_trace.on || g_trace.n >= g_trace.cap) return;
+        slot = g_trace.n++;
+        g_trace.kid[slot] = k;
+        g_trace.flops[slot] = fl;
+        g_trace.bytes[slot] = by;
+        cudaEventRecord(g_trace.ev[2 * slot], s);
+    }
+    ~TraceScope() {
+        if (slot >= 0) cudaEventRecord(g_trace.ev[2 * slot + 1], s);
+    }
+};
 
 constexpr int64_t kMaxGroup = 256;  // widest single TSQR panel group
 constexpr int64_t kMaxLeaf = 256;   // tallest leaf the v1 kernels stage in shared memory
@@ -72,15 +108,80 @@ static inline int64_t merges_at(int64_t L, int level) {
     const int64_t h = int64_t(1) << level;
     return (L - 1 >= h) ? (L - 1 - h) / (2 * h) + 1 : 0;
 }
-static inline size_t group_t_elems(const Geom& G) { return (size_t)2 * G.L * G.npan * kPW * kPW; }
+// Workspace of one panel group: T blocks [2][L][npan][32][32] (leaf T's, then
+// merge T's indexed by the merge's right member), then the fused kernel's
+// ticket + per-(slot, panel) ready flags.
+static inline size_t group_t_bytes(const Geom& G, size_t es) {
+    return (size_t)2 * G.L * G.npan * kPW * kPW * es;
+}
+static inline size_t group_sync_bytes(const Geom& G) {
+    return (size_t)round_up((32 + G.L * G.npan) * (int64_t)sizeof(int), 256);
+}
+static inline size_t group_ws_bytes(const Geom& G, size_t es) {
+    return group_t_bytes(G, es) + group_sync_bytes(G);
+}
 
 static size_t plan_ws_bytes(const Plan& pl) {
-    size_t elems = 0;
-    for (int64_t g = 0; g < pl.ngroups; ++g) elems += group_t_elems(group_geom(pl, g, pl.m));
-    return elems * (pl.dtype == CAQR_F64 ? 8 : 4);
+    size_t bytes = 0;
+    const size_t es = pl.dtype == CAQR_F64 ? 8 : 4;
+    for (int64_t g = 0; g < pl.ngroups; ++g) bytes += group_ws_bytes(group_geom(pl, g, pl.m), es);
+    return bytes;
+}
+
+// Can the persistent fused kernel take this group?  Every task's gathered rows
+// must fit its 256-row register layout: leaves (b rows) and merges (2 wp + 32 p).
+static bool fused_ok(const Geom& G) {
+    if (G.b > kFusedMaxRows) return false;
+    for (int p = 0; p < G.npan; ++p) {
+        const int wp = std::min<int>(kPW, G.ncols - 32 * p);
+        if (2 * wp + 32 * p > kFusedMaxRows) return false;
+    }
+    return true;
+}
+static int num_sms() {
+    static int cache[64] = {};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 64 && cache[dev]) return cache[dev];
+    int n = 148;
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    if (dev < 64) cache[dev] = n;
+    return n;
 }
 
 // ---- launch helpers ---------------------------------------------------------
+
+// Host replica of node_rows()'s gathered-row count (trace bookkeeping only).
+static int64_t node_rg(const Geom& G, int level, int64_t node, int p, int wp) {
+    if (level < 0) {
+        const int64_t h = std::min(G.b, G.mrows - node * G.b);
+        return std::max<int64_t>(0, h - 32 * p);
+    }
+    const int64_t a = node << (level + 1), bb = a + (int64_t(1) << level);
+    const int64_t hb = std::min(G.b, G.mrows - bb * G.b);
+    return wp + std::min<int64_t>(32 * p + wp, hb);
+}
+// Algorithmic work of one launch: Householder QR of each node's gathered
+// RG x wp panel (LAPACK count) / the two GEMMs of the blocked update
+// (4 RG wp ccount); bytes = the panel / C block read and written once (+ V).
+static void trace_counts(const Geom& G, int level, int p, int64_t nodes, bool update,
+                         int64_t ccount, size_t es, double* fl, double* by) {
+    *fl = 0;
+    *by = 0;
+    if (!g_trace.on) return;
+    const int wp = std::min<int>(kPW, G.ncols - 32 * p);
+    for (int64_t nd = 0; nd < nodes; ++nd) {
+        const double rg = (double)node_rg(G, level, nd, p, wp);
+        const double k = std::min<double>(rg, wp);
+        if (!update) {
+            *fl += 2.0 * rg * wp * k - 2.0 / 3.0 * k * k * k;
+            *by += 2.0 * rg * wp * es;
+        } else {
+            *fl += 4.0 * rg * wp * ccount;
+            *by += (2.0 * rg * ccount + rg * wp) * es;
+        }
+    }
+}
 // Opt a kernel into > 48 KB of dynamic shared memory, once per (kernel, device).
 static cudaError_t allow_smem_ptr(const void* kernel, size_t bytes) {
     if (bytes <= 48 * 1024) return cudaSuccess;
@@ -95,8 +196,12 @@ static cudaError_t allow_smem_ptr(const void* kernel, size_t bytes) {
         if (keys[i] == kernel && devs[i] == dev) return cudaSuccess;
     int optin = 0;
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-    if ((size_t)optin < bytes) return cudaErrorInvalidValue;
-    cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, optin);
+    cudaFuncAttributes fa;
+    cudaError_t e = cudaFuncGetAttributes(&fa, kernel);
+    if (e != cudaSuccess) return e;
+    const int maxdyn = optin - (int)fa.sharedSizeBytes;
+    if (maxdyn < (int)bytes) return cudaErrorInvalidValue;
+    e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, maxdyn);
     if (e == cudaSuccess && nkeys < 256) {
         keys[nkeys] = kernel;
         devs[nkeys] = dev;
@@ -117,6 +222,9 @@ static int launch_factor(const Geom& G, T* A, T* Tws, int level, int p, int64_t 
     const int rgmax = level < 0 ? (int)std::min<int64_t>(G.b, G.mrows) : 2 * wp + 32 * p;
     const size_t smem = panel_factor_smem<T>(wp, rgmax);
     cudaError_t e = allow_smem(panel_factor_kernel<T>, smem);
+    double fl, by;
+    trace_counts(G, level, p, nodes, false, 0, sizeof(T), &fl, &by);
+    TraceScope ts(K_PANEL_FACTOR, fl, by, s);
     if (e == cudaSuccess) {
         panel_factor_kernel<T><<<dim3((unsigned)nodes), kThreads, smem, s>>>(G, A, Tws, level, p);
         e = cudaGetLastError();
@@ -137,6 +245,9 @@ static int launch_update(const Geom& G, const T* A, const T* Tws, int level, int
     const int rgmax = level < 0 ? (int)std::min<int64_t>(G.b, G.mrows) : 2 * wp + 32 * p;
     const size_t smem = panel_update_smem<T>(rgmax);
     cudaError_t e = allow_smem(panel_update_kernel<T>, smem);
+    double fl, by;
+    trace_counts(G, level, p, nodes, true, ccount, sizeof(T), &fl, &by);
+    TraceScope ts(K_PANEL_UPDATE, fl, by, s);
     if (e == cudaSuccess) {
         dim3 grid((unsigned)nodes, (unsigned)ceil_div(ccount, 32));
         panel_update_kernel<T><<<grid, kThreads, smem, s>>>(G, A, Tws, level, p, C, ldc, cfirst,
@@ -150,10 +261,53 @@ static int launch_update(const Geom& G, const T* A, const T* Tws, int level, int
     return 0;
 }
 
+// The whole TSQR of a group (leaves + every tree level) in one persistent launch.
+template <typename T>
+static int launch_fused(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, cudaStream_t s) {
+    const int nl = tree_levels(G.L);
+    int64_t total = do_leaves ? G.L : 0;
+    for (int lv = 0; lv < nl; ++lv) total += merges_at(G.L, lv);
+    if (total <= 0) return 0;
+    cudaError_t e = cudaMemsetAsync(sync, 0, group_sync_bytes(G), s);
+    const size_t smem = fused_smem_bytes<T>();
+    if (e == cudaSuccess) e = allow_smem(tsqr_fused_kernel<T>, smem);
+    int occ = 1;
+    if (e == cudaSuccess)
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, tsqr_fused_kernel<T>, kThreads, smem);
+    if (e == cudaSuccess) {
+        const int64_t grid = std::min<int64_t>(total, (int64_t)std::max(occ, 1) * num_sms());
+        double fl = 0, by = 0;
+        if (g_trace.on) {
+            const double mr = (double)G.mrows, nc = (double)G.ncols;
+            fl = do_leaves ? 2.0 * mr * nc * nc - 2.0 / 3.0 * nc * nc * nc
+                           : (double)(G.L - 1) * 2.0 / 3.0 * nc * nc * nc;
+            by = 2.0 * mr * nc * sizeof(T);
+        }
+        TraceScope ts(K_TSQR_FUSED, fl, by, s);
+        tsqr_fused_kernel<T><<<(unsigned)grid, kThreads, smem, s>>>(G, A, Tws, sync, nl, do_leaves ? 1 : 0);
+        e = cudaGetLastError();
+    }
+    if (e != cudaSuccess) {
+        g_last_cuda_error = (int)e;
+        return CAQR_ERR_CUDA;
+    }
+    return 0;
+}
+
+static inline int fused_policy() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = getenv("CAQR_FUSED");
+        v = (e && e[0] == '0') ? 0 : 1;
+    }
+    return v;
+}
+
 // TSQR of one panel group (Fig. 4 minus the trailing update): every leaf's
 // panels (factor + intra-group trailing update), then every tree level.
 template <typename T>
-static int factor_group(const Geom& G, T* A, T* Tws, bool do_leaves, cudaStream_t s) {
+static int factor_group(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, cudaStream_t s) {
+    if (fused_policy() && fused_ok(G)) return launch_fused<T>(G, A, Tws, sync, do_leaves, s);
     int rc = 0;
     if (do_leaves) {
         for (int p = 0; p < G.npan && !rc; ++p) {
@@ -208,6 +362,7 @@ template <typename T>
 static int launch_extract_r(int64_t n, const T* A, int64_t lda, T* R, int64_t ldr, cudaStream_t s) {
     if (n <= 0) return 0;
     dim3 grid((unsigned)std::min<int64_t>(ceil_div(n, 256), 64), (unsigned)n);
+    TraceScope ts(K_EXTRACT_R, 0.0, 2.0 * n * n * sizeof(T), s);
     extract_r_kernel<T><<<grid, 256, 0, s>>>(n, A, lda, R, ldr);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) {
@@ -233,14 +388,16 @@ static int factor_impl(int64_t m, int64_t n, T* A, int64_t lda, T* R, int64_t ld
     if (m == 0 || n == 0) return 0;
     if (!ws) return -7;
     if (ws_bytes < plan_ws_bytes(pl)) return -8;
-    T* Tws = static_cast<T*>(ws);
+    char* wsb = static_cast<char*>(ws);
     for (int64_t g = 0; g < pl.ngroups && !rc; ++g) {
         const Geom G = group_geom(pl, g, lda);
-        rc = factor_group<T>(G, A, Tws, true, s);
+        T* Tws = reinterpret_cast<T*>(wsb);
+        int* sync = reinterpret_cast<int*>(wsb + group_t_bytes(G, sizeof(T)));
+        rc = factor_group<T>(G, A, Tws, sync, true, s);
         const int64_t trail0 = G.col0 + G.ncols;
         if (!rc && trail0 < n)  // CAQR trailing update
             rc = apply_group<T>(G, A, Tws, true, A, lda, trail0, n - trail0, 1, s);
-        Tws += group_t_elems(G);
+        wsb += group_ws_bytes(G, sizeof(T));
     }
     if (!rc) rc = launch_extract_r<T>(n, A, lda, R, ldr, s);
     return rc;
@@ -268,10 +425,10 @@ static int apply_impl(int64_t m, int64_t n, const T* A, int64_t lda, const void*
     int64_t ng = pl.ngroups;
     if (ng > 1024) return CAQR_ERR_UNSUPPORTED;
     {
-        const T* t = base;
+        const char* t = reinterpret_cast<const char*>(base);
         for (int64_t g = 0; g < ng; ++g) {
-            tws[g] = t;
-            t += group_t_elems(group_geom(pl, g, lda));
+            tws[g] = reinterpret_cast<const T*>(t);
+            t += group_ws_bytes(group_geom(pl, g, lda), sizeof(T));
         }
     }
     if (trans) {
@@ -296,8 +453,12 @@ static int form_q_impl(int64_t m, int64_t n, const T* A, int64_t lda, const void
     if (m == 0 || n == 0) return 0;
     if (!ws) return -5;
     dim3 grid((unsigned)std::min<int64_t>(ceil_div(m, 256), 1024), (unsigned)n);
-    set_identity_kernel<T><<<grid, 256, 0, s>>>(m, n, Q, ldq);
-    cudaError_t e = cudaGetLastError();
+    cudaError_t e;
+    {
+        TraceScope ts(K_SET_IDENTITY, 0.0, (double)m * n * sizeof(T), s);
+        set_identity_kernel<T><<<grid, 256, 0, s>>>(m, n, Q, ldq);
+        e = cudaGetLastError();
+    }
     if (e != cudaSuccess) {
         g_last_cuda_error = (int)e;
         return CAQR_ERR_CUDA;
@@ -333,7 +494,8 @@ static int combine_impl(int P, int64_t n, T* Rs, int64_t ld, T* R, int64_t ldr, 
     if (!ws) return -7;
     if (ws_bytes < caqr_combine_workspace_bytes(P, n, dtype)) return -8;
     const Geom G = combine_geom(P, n, ld);
-    int rc = factor_group<T>(G, Rs, static_cast<T*>(ws), false, s);
+    int* sync = reinterpret_cast<int*>(static_cast<char*>(ws) + group_t_bytes(G, sizeof(T)));
+    int rc = factor_group<T>(G, Rs, static_cast<T*>(ws), sync, false, s);
     if (!rc) rc = launch_extract_r<T>(n, Rs, ld, R, ldr, s);
     return rc;
 }
@@ -407,8 +569,8 @@ size_t caqr_combine_workspace_bytes(int P, int64_t n, int dtype) {
     const Geom G = combine_geom(P, n, (int64_t)P * n);
     // T blocks + room for P contiguous n x n blocks (the NCCL receive buffer of
     // caqr_dist_factor_*).
-    const size_t elems = group_t_elems(G) + (size_t)P * n * n;
-    return elems * (dtype == CAQR_F64 ? 8 : 4);
+    const size_t es = dtype == CAQR_F64 ? 8 : 4;
+    return group_ws_bytes(G, es) + (size_t)P * n * n * es;
 }
 int caqr_combine_f32(int P, int64_t n, float* Rs, int64_t ld, float* R, int64_t ldr, void* ws,
                      size_t ws_bytes, caqr_stream_t stream) {
@@ -436,6 +598,52 @@ const char* caqr_strerror(int info) {
     return "unknown";
 }
 int caqr_last_cuda_error(void) { return g_last_cuda_error; }
+
+int caqr_trace_begin(int capacity) {
+    if (capacity < 1) return -1;
+    std::lock_guard<std::mutex> lk(g_trace.mu);
+    if (g_trace.on) return -2;
+    if (g_trace.cap < capacity) {
+        for (int i = 0; i < 2 * g_trace.cap; ++i) cudaEventDestroy(g_trace.ev[i]);
+        delete[] g_trace.ev;
+        delete[] g_trace.kid;
+        delete[] g_trace.flops;
+        delete[] g_trace.bytes;
+        g_trace.ev = new cudaEvent_t[2 * capacity];
+        g_trace.kid = new int[capacity];
+        g_trace.flops = new double[capacity];
+        g_trace.bytes = new double[capacity];
+        for (int i = 0; i < 2 * capacity; ++i)
+            if (cudaEventCreate(&g_trace.ev[i]) != cudaSuccess) {
+                g_trace.cap = i / 2;
+                return CAQR_ERR_CUDA;
+            }
+        g_trace.cap = capacity;
+    }
+    g_trace.n = 0;
+    g_trace.on = true;
+    return 0;
+}
+
+int caqr_trace_end(int* kernel_ids, float* ms, double* flops, double* bytes, int cap) {
+    std::lock_guard<std::mutex> lk(g_trace.mu);
+    g_trace.on = false;
+    const int n = std::min(g_trace.n, cap);
+    for (int i = 0; i < n; ++i) {
+        float t = 0.f;
+        if (cudaEventSynchronize(g_trace.ev[2 * i + 1]) != cudaSuccess ||
+            cudaEventElapsedTime(&t, g_trace.ev[2 * i], g_trace.ev[2 * i + 1]) != cudaSuccess)
+            t = -1.f;
+        if (kernel_ids) kernel_ids[i] = g_trace.kid[i];
+        if (ms) ms[i] = t;
+        if (flops) flops[i] = g_trace.flops[i];
+        if (bytes) bytes[i] = g_trace.bytes[i];
+    }
+    return g_trace.n;
+}
+
+const char* caqr_kernel_name(int id) { return (id >= 0 && id < K_NUM) ? kKernelNames[id] : "?"; }
+
 const char* caqr_build_info(void) {
     return "libcaqr: sm_100a TSQR/CAQR (panel_factor + panel_update kernels, FFMA/DFMA), "
            "built " __DATE__ " " __TIME__;

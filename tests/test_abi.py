@@ -35,10 +35,13 @@ def test_sass_is_sm100a():
 
 
 def test_workspace_bytes(L):
-    # one T block (32x32) per (leaf, panel) and per (merge, panel): 2*L*npan*1024 elems
-    assert caqr.caqr_workspace_bytes(4096, 16) == 2 * 16 * 1 * 1024 * 4
-    assert caqr.caqr_workspace_bytes(4096, 16, caqr.CAQR_F64) == 2 * 16 * 1 * 1024 * 8
-    assert caqr.caqr_workspace_bytes(1_000_000, 192) == 2 * 3907 * 6 * 1024 * 4
+    # one T block (32x32) per (leaf, panel) and per (merge, panel): 2*L*npan*1024 elems,
+    # plus the fused kernel's ticket + (slot, panel) flags: (32 + L*npan) ints, 256-B rounded
+    def ws(L, npan, es):
+        return 2 * L * npan * 1024 * es + -(-(32 + L * npan) * 4 // 256) * 256
+    assert caqr.caqr_workspace_bytes(4096, 16) == ws(16, 1, 4)
+    assert caqr.caqr_workspace_bytes(4096, 16, caqr.CAQR_F64) == ws(16, 1, 8)
+    assert caqr.caqr_workspace_bytes(1_000_000, 192) == ws(3907, 6, 4)
     assert caqr.caqr_workspace_bytes(10, 11) == 0  # n > m
     assert caqr.caqr_workspace_bytes(-1, 1) == 0
     assert caqr.caqr_workspace_bytes(10, 2, 7) == 0  # bad dtype

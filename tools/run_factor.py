@@ -1,0 +1,29 @@
+"""Profiling driver: run caqr_factor on an m x n Gaussian a few times (for ncu)."""
+import argparse
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch
+
+from paper_conf_ipps_andersonbdk11_b200 import caqr, workloads
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--m", type=int, default=1_000_000)
+ap.add_argument("--n", type=int, default=192)
+ap.add_argument("--dtype", default="f32")
+ap.add_argument("--reps", type=int, default=2)
+ap.add_argument("--leaf-rows", type=int, default=0)
+ap.add_argument("--apply", action="store_true")
+a = ap.parse_args()
+dt = torch.float32 if a.dtype == "f32" else torch.float64
+A0 = workloads.device_gaussian(a.m, a.n, seed=0, dtype=dt, device="cuda").t()
+A = caqr.colmajor_empty(a.m, a.n, dt)
+opts = caqr.make_opts(a.leaf_rows)
+for _ in range(a.reps):
+    A.copy_(A0)
+    R, ws = caqr.caqr_factor(A, opts=opts)
+    if a.apply:
+        Q = caqr.caqr_form_q(A, ws, opts=opts)
+torch.cuda.synchronize()
+print("done")
