@@ -195,6 +195,12 @@ const char *caqr_build_info(void);       /* "sm_100a ..." */
 int caqr_trace_begin(int capacity);
 int caqr_trace_end(int *kernel_ids, float *ms, double *flops, double *bytes, int cap);
 const char *caqr_kernel_name(int id);
+/* Phase profile of the fused TSQR kernel (only when the process runs with
+ * CAQR_PROFILE=1): per-phase clock64 cycle sums over all CTAs, then reset.
+ * out[0..9] = task fetch, wait for children, stage panel, factor panel, store +
+ * V form, G/T, stage C, V^T C, apply, publish; out[10]/out[11] = leaf / merge
+ * panel-steps.  Returns 0, or -1 when profiling is off. */
+int caqr_debug_profile_read(unsigned long long out[16]);
 
 /* Plan introspection (host only; for tests and the bench's roofline bookkeeping).
  * Fills out[0..7] = {leaf_rows, panel_cols, groups, leaves(group 0),

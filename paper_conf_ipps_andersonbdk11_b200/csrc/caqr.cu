@@ -261,6 +261,20 @@ static int launch_update(const Geom& G, const T* A, const T* Tws, int level, int
     return 0;
 }
 
+// Phase profile of the fused kernel (diagnostics, CAQR_PROFILE=1).
+static unsigned long long* g_prof = nullptr;
+static unsigned long long* prof_buffer() {
+    static int on = -1;
+    if (on < 0) {
+        const char* e = getenv("CAQR_PROFILE");
+        on = (e && e[0] == '1') ? 1 : 0;
+    }
+    if (!on) return nullptr;
+    if (!g_prof && cudaMalloc(&g_prof, 16 * sizeof(unsigned long long)) == cudaSuccess)
+        cudaMemset(g_prof, 0, 16 * sizeof(unsigned long long));
+    return g_prof;
+}
+
 // The whole TSQR of a group (leaves + every tree level) in one persistent launch.
 template <typename T>
 static int launch_fused(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, cudaStream_t s) {
@@ -284,7 +298,8 @@ static int launch_fused(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, 
             by = 2.0 * mr * nc * sizeof(T);
         }
         TraceScope ts(K_TSQR_FUSED, fl, by, s);
-        tsqr_fused_kernel<T><<<(unsigned)grid, kThreads, smem, s>>>(G, A, Tws, sync, nl, do_leaves ? 1 : 0);
+        tsqr_fused_kernel<T><<<(unsigned)grid, kThreads, smem, s>>>(G, A, Tws, sync, nl, do_leaves ? 1 : 0,
+                                                                    prof_buffer());
         e = cudaGetLastError();
     }
     if (e != cudaSuccess) {
@@ -640,6 +655,14 @@ int caqr_trace_end(int* kernel_ids, float* ms, double* flops, double* bytes, int
         if (bytes) bytes[i] = g_trace.bytes[i];
     }
     return g_trace.n;
+}
+
+int caqr_debug_profile_read(unsigned long long out[16]) {
+    if (!g_prof) return -1;
+    cudaDeviceSynchronize();
+    cudaMemcpy(out, g_prof, 16 * sizeof(unsigned long long), cudaMemcpyDeviceToHost);
+    cudaMemset(g_prof, 0, 16 * sizeof(unsigned long long));
+    return 0;
 }
 
 const char* caqr_kernel_name(int id) { return (id >= 0 && id < K_NUM) ? kKernelNames[id] : "?"; }

@@ -18,12 +18,15 @@
 
 namespace caqr {
 
-// Padded column layout of shared tiles: 16 bytes of padding after every 32
-// rows, so that threads owning different 32-row segments of a column (and
-// 16-byte vector loads of 8 different columns) hit disjoint bank groups.
+// Padded column layout of shared tiles, matched to the panel's thread layout
+// (PanelLayout<8>): rows 0..31 plain, then 28-row segments each followed by
+// PADS elements of padding, so the 8 segment owners of a column -- and 16-byte
+// vector loads by lanes at the same offset of different segments -- hit 8
+// different 16-byte bank groups (segment stride = 16 bytes mod 128).
 template <typename T>
 __host__ __device__ __forceinline__ int padr(int r) {
-    return r + (r >> 5) * int(16 / sizeof(T));
+    constexpr int PADS = sizeof(T) == 4 ? 8 : 6;
+    return r < 32 ? r : r + PADS * ((r - 32) / 28);
 }
 // Column stride for tiles of up to `rows` rows: (stride * sizeof(T)) % 128 == 16.
 template <typename T>
@@ -75,118 +78,394 @@ __device__ __forceinline__ T group_sum(T v, unsigned mask) {
     return v;
 }
 
-// ---------------------------------------------------------------------------
-// Factor the staged panel P (RG x wp, padded column layout) in registers.
-// Thread t owns column c = t / TPC and rows [s*SEG, s*SEG+SEG), s = t % TPC.
-// On exit: P holds the stored form (R on/above the diagonal, v below) and
-// tau_s[0..wp) the reflector scalars.
-// ---------------------------------------------------------------------------
+// Row layout of a column's TPC owner threads: the top 32 rows (where every
+// reflector head of the panel lies) are dealt round-robin, TOPR = 32/TPC rows
+// per thread; the remaining rows are contiguous chunks of BULK rows.  Only the
+// TOPR top rows ever need per-row "r > j" logic.
+template <int TPC>
+struct PanelLayout {
+    static constexpr int SEG = kFusedMaxRows / TPC;
+    static constexpr int TOPR = 32 / TPC;
+    static constexpr int BULK = SEG - TOPR;
+    __device__ static __forceinline__ int row(int s, int i) {
+        return i < TOPR ? s + TPC * i : 32 + BULK * s + (i - TOPR);
+    }
+};
+
 template <typename T, int TPC>
-__device__ __forceinline__ void factor_panel_regs(T* P, int RGP, int RG, int wp, T* tau_s) {
-    constexpr int SEG = kFusedMaxRows / TPC;
-    static_assert(SEG % 4 == 0, "SEG");
+__device__ __forceinline__ void load_col(const T* col, int s, T (&x)[PanelLayout<TPC>::SEG]) {
+    using Lay = PanelLayout<TPC>;
     using V4 = typename Vec4<T>::type;
     constexpr int VN = Vec4<T>::n;
-    const int t = threadIdx.x;
-    const int c = t / TPC, s = t % TPC, r0 = s * SEG;
-    const int lane = t & 31;
-    const unsigned gmask = TPC == 32 ? 0xffffffffu : (((1u << TPC) - 1u) << (lane & ~(TPC - 1)));
-    const bool active = c < wp;
-    T x[SEG];
-    {
-        const T* pc = P + (size_t)min(c, 31) * RGP + padr<T>(r0);
 #pragma unroll
-        for (int i = 0; i < SEG; i += VN) {
-            const V4 q = *reinterpret_cast<const V4*>(pc + i);
+    for (int i = 0; i < Lay::TOPR; ++i) x[i] = col[padr<T>(s + TPC * i)];
+    if constexpr (Lay::BULK % 4 == 0) {
 #pragma unroll
-            for (int k = 0; k < VN; ++k) x[i + k] = (active && r0 + i + k < RG) ? vget<T>(q, k) : T(0);
+        for (int i = 0; i < Lay::BULK; i += VN) {
+            const V4 q = *reinterpret_cast<const V4*>(col + padr<T>(32 + Lay::BULK * s + i));
+#pragma unroll
+            for (int k = 0; k < VN; ++k) x[Lay::TOPR + i + k] = vget<T>(q, k);
         }
+    } else {
+#pragma unroll
+        for (int i = 0; i < Lay::BULK; ++i) x[Lay::TOPR + i] = col[padr<T>(32 + Lay::BULK * s + i)];
     }
-    __syncthreads();  // everyone has its registers before P is overwritten with v's
+}
 
-    // Reflector of column j by its owner group (xLARFG, reading S1).  Writes the
-    // v column (unit head, zeros above) into P[:, j] for the other groups.
-    auto reflector = [&](int j) {
-        T sig = T(0), al = T(0);
+template <typename T, int TPC>
+__device__ __forceinline__ void store_col(T* col, int s, const T (&x)[PanelLayout<TPC>::SEG]) {
+    using Lay = PanelLayout<TPC>;
+    using V4 = typename Vec4<T>::type;
+    constexpr int VN = Vec4<T>::n;
 #pragma unroll
-        for (int i = 0; i < SEG; ++i) {
-            const int r = r0 + i;
-            sig = (r > j) ? fma(x[i], x[i], sig) : sig;
-            al = (r == j) ? x[i] : al;
-        }
-        sig = group_sum<TPC>(sig, gmask);
-        al = group_sum<TPC>(al, gmask);
-        T tau = T(0), beta = al, scale = T(0);
-        if (j < RG && sig != T(0)) {
-            const T mu = sqrt(fma(al, al, sig));
-            beta = -copysign(mu, al);
-            tau = (beta - al) / beta;
-            scale = T(1) / (al - beta);
-        }
-        T* pj = P + (size_t)j * RGP + padr<T>(r0);
+    for (int i = 0; i < Lay::TOPR; ++i) col[padr<T>(s + TPC * i)] = x[i];
+    if constexpr (Lay::BULK % 4 == 0) {
 #pragma unroll
-        for (int i = 0; i < SEG; i += VN) {
+        for (int i = 0; i < Lay::BULK; i += VN) {
             V4 q;
             T* qq = reinterpret_cast<T*>(&q);
 #pragma unroll
-            for (int k = 0; k < VN; ++k) {
-                const int r = r0 + i + k;
-                if (r > j) x[i + k] = (tau != T(0)) ? x[i + k] * scale : x[i + k];
-                if (r == j) x[i + k] = beta;
-                qq[k] = r > j ? x[i + k] : (r == j ? T(1) : T(0));
-            }
-            *reinterpret_cast<V4*>(pj + i) = q;
+            for (int k = 0; k < VN; ++k) qq[k] = x[Lay::TOPR + i + k];
+            *reinterpret_cast<V4*>(col + padr<T>(32 + Lay::BULK * s + i)) = q;
         }
+    } else {
+#pragma unroll
+        for (int i = 0; i < Lay::BULK; ++i) col[padr<T>(32 + Lay::BULK * s + i)] = x[Lay::TOPR + i];
+    }
+}
+
+// ---------------------------------------------------------------------------
+// Factor the staged panel P (RG x wp, padded column layout) in registers.
+// Thread t owns column c = t / TPC (rows per PanelLayout, s = t % TPC).
+// On exit: P holds the stored form (R on/above the diagonal, v below) and
+// tau_s[0..wp) the reflector scalars.
+// All warp shuffles run with the full mask in warp-uniform control flow (a
+// partial mask under divergence compiles to slow WARPSYNC.COLLECTIVE code);
+// groups that have nothing to do compute on zeros and discard.
+// ---------------------------------------------------------------------------
+template <typename T>
+__device__ __forceinline__ T rcp_rn(T x) {
+    if constexpr (sizeof(T) == 4)
+        return __frcp_rn(x);
+    else
+        return __drcp_rn(x);
+}
+
+// 1/sqrt(s) and sqrt(s), s > 0.  fp32: hardware approximations plus one
+// Newton step (~1 ulp; the reflector stays orthogonal to that level), far
+// cheaper on the critical path than the IEEE-rounded sqrt / division
+// subroutines.  fp64: IEEE-rounded.
+template <typename T>
+__device__ __forceinline__ void rsqrt_refined(T s, T& r, T& sq) {
+    if constexpr (sizeof(T) == 4) {
+        float y = rsqrtf(s);
+        const float h = 0.5f * s * y;
+        y = fmaf(-h, y, 1.5f) * y;  // y (1.5 - 0.5 s y^2)
+        r = y;
+        const float q = s * y;      // sqrt(s) ~ s / sqrt(s), one residual correction
+        sq = fmaf(fmaf(-q, q, s), 0.5f * y, q);
+    } else {
+        sq = sqrt(s);
+        r = __drcp_rn(sq);
+    }
+}
+template <typename T>
+__device__ __forceinline__ T rcp_refined(T d) {
+    if constexpr (sizeof(T) == 4) {
+        float y = __fdividef(1.0f, d);
+        return fmaf(fmaf(-d, y, 1.0f), y, y);  // one Newton step
+    } else {
+        return __drcp_rn(d);
+    }
+}
+
+template <typename T, int TPC>
+__device__ __forceinline__ void factor_panel_regs(T* P, int RGP, int RG, int wp, T* tau_s) {
+    using Lay = PanelLayout<TPC>;
+    constexpr int SEG = Lay::SEG, TOPR = Lay::TOPR;
+    constexpr int GPW = 32 / TPC;  // column groups per warp
+    const int t = threadIdx.x;
+    const int c = t / TPC, s = t % TPC;
+    const int warp = t >> 5;
+    const bool active = c < wp;
+    T x[SEG];
+    load_col<T, TPC>(P + (size_t)min(c, 31) * RGP, s, x);
+#pragma unroll
+    for (int i = 0; i < SEG; ++i)
+        if (!(active && Lay::row(s, i) < RG)) x[i] = T(0);
+    __syncthreads();  // everyone has its registers before P is overwritten with v's
+
+    // Reflector of column j (< 32), run by the whole warp that holds column j
+    // (xLARFG, reading S1): beta = -copysign(mu, alpha), tau = 1 + |alpha|/mu
+    // == (beta-alpha)/beta, scale = copysign(1/(|alpha|+mu), alpha) == 1/(alpha-beta).
+    // The owner group writes v (unit head, zeros above) into P[:, j].
+    auto reflector = [&](int j) {
+        T s0 = 0, s1 = 0, s2 = 0, s3 = 0, al = 0;
+#pragma unroll
+        for (int i = 0; i < TOPR; ++i) {
+            const int r = s + TPC * i;
+            s0 = (r > j) ? fma(x[i], x[i], s0) : s0;
+            al = (r == j) ? x[i] : al;
+        }
+#pragma unroll
+        for (int i = TOPR; i < SEG; i += 4) {
+            s0 = fma(x[i], x[i], s0);
+            if (i + 1 < SEG) s1 = fma(x[i + 1], x[i + 1], s1);
+            if (i + 2 < SEG) s2 = fma(x[i + 2], x[i + 2], s2);
+            if (i + 3 < SEG) s3 = fma(x[i + 3], x[i + 3], s3);
+        }
+        T sig = (s0 + s1) + (s2 + s3);
+#pragma unroll
+        for (int o = 1; o < TPC; o <<= 1) {
+            sig += __shfl_xor_sync(0xffffffffu, sig, o);
+            al += __shfl_xor_sync(0xffffffffu, al, o);
+        }
+        if (c != j) return;
+        T tau = T(0), beta = al, scale = T(1);
+        if (j < RG && sig != T(0)) {
+            const T ss = fma(al, al, sig);
+            const T aa = fabs(al);
+            T rmu, mu;
+            rsqrt_refined(ss, rmu, mu);  // 1/mu and mu = sqrt(alpha^2 + sigma)
+            beta = -copysign(mu, al);
+            tau = fma(aa, rmu, T(1));
+            scale = copysign(rcp_refined(aa + mu), al);
+        }
+#pragma unroll
+        for (int i = 0; i < TOPR; ++i) {
+            const int r = s + TPC * i;
+            if (r > j) x[i] *= scale;
+            if (r == j) x[i] = beta;
+        }
+#pragma unroll
+        for (int i = TOPR; i < SEG; ++i) x[i] *= scale;
+        T v[SEG];
+#pragma unroll
+        for (int i = 0; i < SEG; ++i) v[i] = x[i];
+#pragma unroll
+        for (int i = 0; i < TOPR; ++i) {
+            const int r = s + TPC * i;
+            v[i] = r > j ? x[i] : (r == j ? T(1) : T(0));
+        }
+        store_col<T, TPC>(P + (size_t)j * RGP, s, v);
         if (s == 0) tau_s[j] = tau;
     };
 
-    if (c == 0) reflector(0);
+    if (warp == 0) reflector(0);
     __syncthreads();
     for (int j = 0; j < wp; ++j) {
         const T tau = tau_s[j];
-        if (active && c > j) {
-            if (tau != T(0)) {
-                const T* pj = P + (size_t)j * RGP + padr<T>(r0);
-                T d0 = 0, d1 = 0, d2 = 0, d3 = 0;
+        if (warp >= (j + 1) / GPW && tau != T(0)) {  // warps that own some column > j
+            T v[SEG];
+            load_col<T, TPC>(P + (size_t)j * RGP, s, v);
+            T d0 = 0, d1 = 0, d2 = 0, d3 = 0;
 #pragma unroll
-                for (int i = 0; i < SEG; i += 4) {
-                    T v4[4];
-#pragma unroll
-                    for (int h = 0; h < 4 / VN; ++h) {
-                        const V4 q = *reinterpret_cast<const V4*>(pj + i + h * VN);
-#pragma unroll
-                        for (int k = 0; k < VN; ++k) v4[h * VN + k] = vget<T>(q, k);
-                    }
-                    d0 = fma(v4[0], x[i + 0], d0);
-                    d1 = fma(v4[1], x[i + 1], d1);
-                    d2 = fma(v4[2], x[i + 2], d2);
-                    d3 = fma(v4[3], x[i + 3], d3);
-                }
-                T d = group_sum<TPC>((d0 + d1) + (d2 + d3), gmask);
+            for (int i = 0; i < SEG; i += 4) {
+                d0 = fma(v[i], x[i], d0);
+                if (i + 1 < SEG) d1 = fma(v[i + 1], x[i + 1], d1);
+                if (i + 2 < SEG) d2 = fma(v[i + 2], x[i + 2], d2);
+                if (i + 3 < SEG) d3 = fma(v[i + 3], x[i + 3], d3);
+            }
+            const T d = group_sum<TPC>((d0 + d1) + (d2 + d3), 0xffffffffu);
+            if (active && c > j) {
                 const T st = tau * d;
 #pragma unroll
-                for (int i = 0; i < SEG; i += VN) {
-                    const V4 q = *reinterpret_cast<const V4*>(pj + i);
-#pragma unroll
-                    for (int k = 0; k < VN; ++k) x[i + k] = fma(-st, vget<T>(q, k), x[i + k]);
-                }
+                for (int i = 0; i < SEG; ++i) x[i] = fma(-st, v[i], x[i]);
             }
-            if (c == j + 1) reflector(j + 1);
         }
+        if (j + 1 < wp && warp == (j + 1) / GPW) reflector(j + 1);
         __syncthreads();
     }
     // stored form back into P (R on/above the diagonal, v below)
-    if (active) {
-        T* pc = P + (size_t)c * RGP + padr<T>(r0);
+    if (active) store_col<T, TPC>(P + (size_t)c * RGP, s, x);
+    __syncthreads();
+}
+
+// ---------------------------------------------------------------------------
+// Panel factorization, 4-column blocks ("WB4").  Warp w owns panel columns
+// 4w..4w+3; lane l holds rows l + 32 i (i < 8) of each of them in registers
+// (every reflector head, row j < 32, sits in lane j, i = 0).  Block b: warp b
+// computes its 4 reflectors warp-locally (shuffle reductions only, no CTA
+// barrier), publishes v (V form) into P and its 4x4 compact-WY factor, one CTA
+// barrier, then every warp to the right applies the block as
+// X <- X - V (T^T (V^T X)) to its own 4 columns.  8 barriers per 32 columns.
+// On exit P holds the stored form (R on/above the diagonal, v below) and
+// tau_s[0..wp) the reflector scalars.
+// ---------------------------------------------------------------------------
+template <typename T>
+__device__ __forceinline__ void factor_panel_wb4(T* P, int RGP, int RG, int wp, T* tau_s, T* Tb) {
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int cb = 4 * warp;
+    const int nc = max(0, min(4, wp - cb));
+    T x[4][8];
 #pragma unroll
-        for (int i = 0; i < SEG; i += VN) {
-            V4 q;
-            T* qq = reinterpret_cast<T*>(&q);
+    for (int q = 0; q < 4; ++q)
 #pragma unroll
-            for (int k = 0; k < VN; ++k) qq[k] = x[i + k];
-            *reinterpret_cast<V4*>(pc + i) = q;
+        for (int i = 0; i < 8; ++i) {
+            const int r = lane + 32 * i;
+            x[q][i] = (q < nc && r < RG) ? P[(size_t)(cb + q) * RGP + padr<T>(r)] : T(0);
+        }
+    __syncthreads();  // all columns are in registers before P gets v's
+    const int nblk = (wp + 3) / 4;
+    for (int b = 0; b < nblk; ++b) {
+        if (warp == b) {
+            T tq[4] = {T(0), T(0), T(0), T(0)};
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                if (q < nc) {
+                    const int j = cb + q;
+                    T sg = T(0);
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) {
+                        const int r = lane + 32 * i;
+                        sg = (r > j) ? fma(x[q][i], x[q][i], sg) : sg;
+                    }
+                    const T al = __shfl_sync(0xffffffffu, x[q][0], j);
+                    sg = warp_sum(sg);
+                    T tau = T(0), beta = al, scale = T(1);
+                    if (j < RG && sg != T(0)) {
+                        const T ss = fma(al, al, sg);
+                        const T aa = fabs(al);
+                        T rmu, mu;
+                        rsqrt_refined(ss, rmu, mu);
+                        beta = -copysign(mu, al);
+                        tau = fma(aa, rmu, T(1));
+                        scale = copysign(rcp_refined(aa + mu), al);
+                    }
+                    tq[q] = tau;
+                    T v[8];
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) {
+                        const int r = lane + 32 * i;
+                        if (r > j) x[q][i] *= scale;
+                        if (r == j) x[q][i] = beta;
+                        v[i] = r > j ? x[q][i] : (r == j ? T(1) : T(0));
+                        P[(size_t)j * RGP + padr<T>(r)] = v[i];
+                    }
+                    if (lane == 0) tau_s[j] = tau;
+                    // apply H_j to this warp's later columns (interleaved reductions)
+                    if (tau != T(0)) {
+                        T d[4] = {T(0), T(0), T(0), T(0)};
+#pragma unroll
+                        for (int q2 = q + 1; q2 < 4; ++q2)
+#pragma unroll
+                            for (int i = 0; i < 8; ++i) d[q2] = fma(v[i], x[q2][i], d[q2]);
+#pragma unroll
+                        for (int o = 16; o > 0; o >>= 1)
+#pragma unroll
+                            for (int q2 = q + 1; q2 < 4; ++q2) d[q2] += __shfl_xor_sync(0xffffffffu, d[q2], o);
+#pragma unroll
+                        for (int q2 = q + 1; q2 < 4; ++q2) {
+                            const T st = tau * d[q2];
+#pragma unroll
+                            for (int i = 0; i < 8; ++i) x[q2][i] = fma(-st, v[i], x[q2][i]);
+                        }
+                    }
+                }
+            }
+            // 4x4 compact-WY factor of the block: g_ab = v_a . v_b (a < b), then
+            // T[a][a] = tau_a, T[a][b] = -tau_b sum_{k=a}^{b-1} T[a][k] g_kb.
+            T gv[6];
+            {
+                T vv[4][8];
+#pragma unroll
+                for (int q = 0; q < 4; ++q)
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) {
+                        const int r = lane + 32 * i, j = cb + q;
+                        vv[q][i] = (q < nc) ? (r > j ? x[q][i] : (r == j ? T(1) : T(0))) : T(0);
+                    }
+                int e = 0;
+#pragma unroll
+                for (int a = 0; a < 4; ++a)
+#pragma unroll
+                    for (int bb = a + 1; bb < 4; ++bb, ++e) {
+                        T g = T(0);
+#pragma unroll
+                        for (int i = 0; i < 8; ++i) g = fma(vv[a][i], vv[bb][i], g);
+                        gv[e] = g;
+                    }
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1)
+#pragma unroll
+                    for (int k = 0; k < 6; ++k) gv[k] += __shfl_xor_sync(0xffffffffu, gv[k], o);
+            }
+            if (lane == 0) {
+                // gv index of (a, bb), a < bb: 0:(0,1) 1:(0,2) 2:(0,3) 3:(1,2) 4:(1,3) 5:(2,3)
+                T tm[4][4];
+#pragma unroll
+                for (int a = 0; a < 4; ++a)
+#pragma unroll
+                    for (int bb = 0; bb < 4; ++bb) tm[a][bb] = T(0);
+#pragma unroll
+                for (int a = 0; a < 4; ++a) tm[a][a] = tq[a];
+                const T g01 = gv[0], g02 = gv[1], g03 = gv[2], g12 = gv[3], g13 = gv[4], g23 = gv[5];
+                tm[0][1] = -tq[1] * (tm[0][0] * g01);
+                tm[0][2] = -tq[2] * (tm[0][0] * g02 + tm[0][1] * g12);
+                tm[1][2] = -tq[2] * (tm[1][1] * g12);
+                tm[0][3] = -tq[3] * (tm[0][0] * g03 + tm[0][1] * g13 + tm[0][2] * g23);
+                tm[1][3] = -tq[3] * (tm[1][1] * g13 + tm[1][2] * g23);
+                tm[2][3] = -tq[3] * (tm[2][2] * g23);
+#pragma unroll
+                for (int a = 0; a < 4; ++a)
+#pragma unroll
+                    for (int bb = 0; bb < 4; ++bb) Tb[b * 16 + a * 4 + bb] = tm[a][bb];
+            }
+        }
+        __syncthreads();
+        if (warp > b && nc > 0) {
+            // X <- X - V_b (T_b^T (V_b^T X)) on this warp's columns
+            T vb[4][8];
+            const int jb = 4 * b;
+#pragma unroll
+            for (int a = 0; a < 4; ++a)
+#pragma unroll
+                for (int i = 0; i < 8; ++i) vb[a][i] = P[(size_t)(jb + a) * RGP + padr<T>(lane + 32 * i)];
+            T w[4][4];
+#pragma unroll
+            for (int a = 0; a < 4; ++a)
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    T acc = T(0);
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) acc = fma(vb[a][i], x[q][i], acc);
+                    w[a][q] = acc;
+                }
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1)
+#pragma unroll
+                for (int a = 0; a < 4; ++a)
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) w[a][q] += __shfl_xor_sync(0xffffffffu, w[a][q], o);
+            T tt[16];
+#pragma unroll
+            for (int k = 0; k < 16; ++k) tt[k] = Tb[b * 16 + k];
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                T w2[4];
+#pragma unroll
+                for (int a = 0; a < 4; ++a) {
+                    T acc = T(0);
+#pragma unroll
+                    for (int k = 0; k <= a; ++k) acc = fma(tt[k * 4 + a], w[k][q], acc);
+                    w2[a] = acc;
+                }
+#pragma unroll
+                for (int i = 0; i < 8; ++i) {
+                    T xv = x[q][i];
+#pragma unroll
+                    for (int a = 0; a < 4; ++a) xv = fma(-vb[a][i], w2[a], xv);
+                    x[q][i] = xv;
+                }
+            }
         }
     }
+    __syncthreads();  // every block applied: P's v columns are no longer read
+#pragma unroll
+    for (int q = 0; q < 4; ++q)
+        if (q < nc)
+#pragma unroll
+            for (int i = 0; i < 8; ++i) P[(size_t)(cb + q) * RGP + padr<T>(lane + 32 * i)] = x[q][i];
     __syncthreads();
 }
 
@@ -239,9 +518,10 @@ __device__ __forceinline__ void gemm_vtc(const T* Vs, const T* Cs, int RGP, int 
     __syncthreads();
 }
 
-// T (upper triangular, Tt[r*kTS+c] = T[r][c]) from G = V^T V (in G) and tau
-// (xLARFT forward/columnwise): T[j][j] = tau_j, T[0:j,j] = -tau_j T[0:j,0:j] G[0:j,j].
-// One warp; lane i keeps row i of T in registers.
+// T (upper triangular, Tt[r*kTS+c] = T[r][c]) from G = V^T V (strict upper
+// part in G) and tau (xLARFT forward/columnwise): T[j][j] = tau_j,
+// T[0:j,j] = -tau_j T[0:j,0:j] G[0:j,j].  One warp; lane i keeps row i of T in
+// registers; 4 independent accumulation chains.
 template <typename T>
 __device__ __forceinline__ void build_t(const T* G, const T* tau_s, int wp, T* Tt) {
     const int lane = threadIdx.x & 31;
@@ -249,18 +529,18 @@ __device__ __forceinline__ void build_t(const T* G, const T* tau_s, int wp, T* T
     T row[32];
 #pragma unroll
     for (int j = 0; j < 32; ++j) {
-        T tj = T(0);
-        if (j < wp) {
-            T a0 = 0, a1 = 0;
+        T a0 = 0, a1 = 0, a2 = 0, a3 = 0;
 #pragma unroll
-            for (int k = 0; k < j; k += 2) {
-                a0 = fma(row[k], G[k * kTS + j], a0);
-                if (k + 1 < j) a1 = fma(row[k + 1], G[(k + 1) * kTS + j], a1);
-            }
-            const T tau = tau_s[j];
-            tj = (j == lane) ? tau : (j > lane ? -tau * (a0 + a1) : T(0));
+        for (int k = 0; k + 3 < j; k += 4) {
+            a0 = fma(row[k + 0], G[(k + 0) * kTS + j], a0);
+            a1 = fma(row[k + 1], G[(k + 1) * kTS + j], a1);
+            a2 = fma(row[k + 2], G[(k + 2) * kTS + j], a2);
+            a3 = fma(row[k + 3], G[(k + 3) * kTS + j], a3);
         }
-        row[j] = tj;
+#pragma unroll
+        for (int k = j & ~3; k < j; ++k) a0 = fma(row[k], G[k * kTS + j], a0);
+        const T tau = j < wp ? tau_s[j] : T(0);
+        row[j] = (j == lane) ? tau : (j > lane ? -tau * ((a0 + a1) + (a2 + a3)) : T(0));
     }
 #pragma unroll
     for (int j = 0; j < 32; ++j) Tt[lane * kTS + j] = row[j];
@@ -274,25 +554,39 @@ __device__ __forceinline__ void apply_block(const T* Vs, const T* Cs, const T* T
     using V4 = typename Vec4<T>::type;
     constexpr int VN = Vec4<T>::n;
     const int tid = threadIdx.x;
+    // W2 = op(T) W: thread (column c, rows jj = jg + 8q); T is zero below its
+    // diagonal, so full unrolled sums need no bounds.
     T w2[4];
+    {
+        const int c = tid & 31, jg = tid >> 5;
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
-        const int e = tid + q * kThreads;
-        const int jj = e >> 5, c = e & 31;
-        T s = T(0);
-        if (trans) {
-            for (int k = 0; k <= jj; ++k) s = fma(Tt[k * kTS + jj], W[k * kTS + c], s);
-        } else {
-            for (int k = jj; k < 32; ++k) s = fma(Tt[jj * kTS + k], W[k * kTS + c], s);
+        for (int q = 0; q < 4; ++q) w2[q] = T(0);
+#pragma unroll
+        for (int h = 0; h < 32; h += 16) {
+            T wc[16];
+#pragma unroll
+            for (int k = 0; k < 16; ++k) wc[k] = W[(h + k) * kTS + c];
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const int jj = jg + 8 * q;
+                T a0 = 0, a1 = 0;
+#pragma unroll
+                for (int k = 0; k < 16; k += 2) {
+                    if (trans) {
+                        a0 = fma(Tt[(h + k) * kTS + jj], wc[k], a0);
+                        a1 = fma(Tt[(h + k + 1) * kTS + jj], wc[k + 1], a1);
+                    } else {
+                        a0 = fma(Tt[jj * kTS + h + k], wc[k], a0);
+                        a1 = fma(Tt[jj * kTS + h + k + 1], wc[k + 1], a1);
+                    }
+                }
+                w2[q] += a0 + a1;
+            }
         }
-        w2[q] = s;
     }
     __syncthreads();
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
-        const int e = tid + q * kThreads;
-        W[(e >> 5) * kTS + (e & 31)] = w2[q];
-    }
+    for (int q = 0; q < 4; ++q) W[((tid >> 5) + 8 * q) * kTS + (tid & 31)] = w2[q];
     __syncthreads();
     const int nq = R32 / 4;
     for (int u = tid; u < nq * 4; u += kThreads) {
@@ -317,40 +611,76 @@ __device__ __forceinline__ void apply_block(const T* Vs, const T* Cs, const T* T
 #pragma unroll
                 for (int k = 0; k < VN; ++k) vr[h * VN + k] = vget<T>(t4, k);
             }
+            T wv[8];
 #pragma unroll
-            for (int c = 0; c < 8; ++c) {
-                const T wv = W[jj * kTS + cbase + c];
+            for (int h = 0; h < 8 / VN; ++h) {
+                const V4 t4 = *reinterpret_cast<const V4*>(W + jj * kTS + cbase + h * VN);
 #pragma unroll
-                for (int i = 0; i < 4; ++i) acc[i][c] = fma(-vr[i], wv, acc[i][c]);
+                for (int k = 0; k < VN; ++k) wv[h * VN + k] = vget<T>(t4, k);
             }
+#pragma unroll
+            for (int c = 0; c < 8; ++c)
+#pragma unroll
+                for (int i = 0; i < 4; ++i) acc[i][c] = fma(-vr[i], wv[c], acc[i][c]);
         }
+        // result back into the staged tile (each element is owned by exactly
+        // this thread), then one coalesced pass to global below
 #pragma unroll
         for (int c = 0; c < 8; ++c) {
-            if (cbase + c >= ncb) break;
-            T* ccol = C + (cb0 + cbase + c) * ldc;
 #pragma unroll
-            for (int i = 0; i < 4; ++i)
-                if (r + i < RG) ccol[gathered_row(nr, r + i)] = acc[i][c];
+            for (int h = 0; h < 4 / VN; ++h) {
+                V4 t4;
+                T* tt = reinterpret_cast<T*>(&t4);
+#pragma unroll
+                for (int k = 0; k < VN; ++k) tt[k] = acc[h * VN + k][c];
+                *reinterpret_cast<V4*>(const_cast<T*>(Cs) + (size_t)(cbase + c) * RGP + pr + h * VN) = t4;
+            }
+        }
+    }
+    __syncthreads();
+    {
+        const int warp = tid >> 5, lane = tid & 31;
+        for (int c = warp; c < ncb; c += kWarps) {
+            T* ccol = C + (cb0 + c) * ldc;
+            const T* cs = Cs + (size_t)c * RGP;
+            for (int r = lane; r < RG; r += 32) ccol[gathered_row(nr, r)] = cs[padr<T>(r)];
         }
     }
     __syncthreads();
 }
 
-// Stage gathered rows of 32 columns [col0, col0+ncol) of M into a padded tile
-// (columns >= ncol and rows >= RG zero).  mask_panel: apply the merge-node
-// structure masks of panel p (panel_entry_stored).
 template <typename T>
 __device__ __forceinline__ void stage_cols(T* S, int RGP, int R32, const T* M, int64_t ld, int64_t col0,
                                            int ncol, const NodeRows& nr, int RG, bool mask_panel, int p) {
+    // Every thread issues all of its loads before the first store (memory-level
+    // parallelism: up to 32 L2/HBM requests in flight per thread), in halves
+    // of 16 for fp64 to bound register use.
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    for (int jj = warp; jj < 32; jj += kWarps) {
-        T* sc = S + (size_t)jj * RGP;
-        const T* mc = M + (col0 + jj) * ld;
-        for (int r = lane; r < R32; r += 32) {
-            T v = T(0);
-            if (jj < ncol && r < RG && (!mask_panel || panel_entry_stored(nr, r, jj, p)))
-                v = ldcg(mc + gathered_row(nr, r));
-            sc[padr<T>(r)] = v;
+    constexpr int NA = sizeof(T) == 4 ? 4 : 2;  // columns per batch per warp
+#pragma unroll
+    for (int a0 = 0; a0 < 4; a0 += NA) {
+        T buf[NA][8];
+#pragma unroll
+        for (int a = 0; a < NA; ++a) {
+            const int jj = warp + 8 * (a0 + a);
+            const T* mc = M + (col0 + jj) * ld;
+#pragma unroll
+            for (int b = 0; b < 8; ++b) {
+                const int r = lane + 32 * b;
+                T v = T(0);
+                if (r < RG && jj < ncol && (!mask_panel || panel_entry_stored(nr, r, jj, p)))
+                    v = ldcg(mc + gathered_row(nr, r));
+                buf[a][b] = v;
+            }
+        }
+#pragma unroll
+        for (int a = 0; a < NA; ++a) {
+            T* sc = S + (size_t)(warp + 8 * (a0 + a)) * RGP;
+#pragma unroll
+            for (int b = 0; b < 8; ++b) {
+                const int r = lane + 32 * b;
+                if (r < R32) sc[padr<T>(r)] = buf[a][b];
+            }
         }
     }
 }
@@ -360,7 +690,8 @@ __device__ __forceinline__ void stage_cols(T* S, int RGP, int R32, const T* M, i
 // ---------------------------------------------------------------------------
 template <typename T>
 __global__ void __launch_bounds__(kThreads, sizeof(T) == 4 ? 2 : 1)
-tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int nlevels, int do_leaves) {
+tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int nlevels, int do_leaves,
+                  unsigned long long* prof) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int RGP = fused_col_stride<T>(kFusedMaxRows);
     T* P = reinterpret_cast<T*>(smem_raw);
@@ -378,8 +709,21 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
         const int64_t h = int64_t(1) << l;
         total += (g.L - 1 >= h) ? (g.L - 1 - h) / (2 * h) + 1 : 0;
     }
+    // optional phase profile (diagnostics; prof == nullptr in normal use)
+    // (accumulators live in shared memory: no registers taken from the math)
+    __shared__ unsigned long long pacc[13];
+    if (threadIdx.x < 13) pacc[threadIdx.x] = threadIdx.x == 12 ? (unsigned long long)clock64() : 0ull;
+#define CAQR_PROF(k)                                              \
+    do {                                                          \
+        if (prof && threadIdx.x == 0) {                           \
+            const unsigned long long t1_ = clock64();             \
+            pacc[k] += t1_ - pacc[12];                            \
+            pacc[12] = t1_;                                       \
+        }                                                         \
+    } while (0)
     for (;;) {
         __syncthreads();
+        CAQR_PROF(0);
         if (threadIdx.x == 0) s_task = atomicAdd(ticket, 1);
         __syncthreads();
         const int64_t task = s_task;
@@ -417,6 +761,8 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
                 while (ld_acquire(fb) < ver_b) __nanosleep(64);
             }
             __syncthreads();
+            CAQR_PROF(1);
+            if (prof && threadIdx.x == 0) pacc[level < 0 ? 10 : 11] += 1;
             const NodeRows nr = node_rows(g, level, node, p, wp);
             const int RG = nr.n0 + nr.n1;
             const int R32 = (RG + 31) & ~31;
@@ -425,10 +771,9 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
             stage_cols(P, RGP, R32, A, g.lda, c0, wp, nr, RG, true, p);
             if (threadIdx.x < 32) tau_s[threadIdx.x] = T(0);
             __syncthreads();
-            if (wp <= 8)
-                factor_panel_regs<T, 32>(P, RGP, RG, wp, tau_s);
-            else
-                factor_panel_regs<T, 8>(P, RGP, RG, wp, tau_s);
+            CAQR_PROF(2);
+            factor_panel_wb4<T>(P, RGP, RG, wp, tau_s, Wp);
+            CAQR_PROF(3);
             {
                 const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
                 for (int jj = warp; jj < wp; jj += kWarps) {
@@ -457,6 +802,7 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
                 }
             }
             __syncthreads();
+            CAQR_PROF(4);
             gemm_vtc(P, P, RGP, R32, Wp, W);  // G = V^T V
             build_t(W, tau_s, wp, Tt);
             __syncthreads();
@@ -467,21 +813,29 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
                     tb[e] = Tt[r * kTS + c];
                 }
             }
+            CAQR_PROF(5);
             // ---- trailing columns of this node, 32 at a time -------------------
             const int64_t tfirst = c0 + 32, tend = g.col0 + g.ncols;
             for (int64_t cb0 = tfirst; cb0 < tend; cb0 += 32) {
                 const int ncb = (int)(tend - cb0 < 32 ? tend - cb0 : 32);
                 stage_cols(Cs, RGP, R32, static_cast<const T*>(A), g.lda, cb0, ncb, nr, RG, false, p);
                 __syncthreads();
+                CAQR_PROF(6);
                 gemm_vtc(P, Cs, RGP, R32, Wp, W);
+                CAQR_PROF(7);
                 apply_block(P, Cs, Tt, W, RGP, R32, RG, wp, 1, nr, A, g.lda, cb0, ncb);
+                CAQR_PROF(8);
             }
             // ---- publish ----------------------------------------------------------
             __threadfence();
             __syncthreads();
             if (threadIdx.x == 0) st_release(flags + slot_a * g.npan + p, level < 0 ? 1 : my_ver);
+            CAQR_PROF(9);
         }
     }
+    if (prof && threadIdx.x == 0)
+        for (int k = 0; k < 12; ++k) atomicAdd(prof + k, pacc[k]);
+#undef CAQR_PROF
 }
 
 }  // namespace caqr

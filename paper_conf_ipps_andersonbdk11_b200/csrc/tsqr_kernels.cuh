@@ -33,7 +33,7 @@ namespace caqr {
 constexpr int kPW = 32;        // max reflectors per panel step (panel width)
 constexpr int kThreads = 256;  // 8 warps
 constexpr int kWarps = kThreads / 32;
-constexpr int kTS = 33;        // stride of 32x32 scratch tiles in shared memory
+constexpr int kTS = 36;        // stride of 32x32 scratch tiles (16-byte aligned rows)
 
 // Geometry of one TSQR panel group (a column panel of width ncols <= 256 that
 // starts at row0 = col0 of A; the grid redrawn "nb rows lower").
