@@ -1,0 +1,108 @@
+"""Row-sharded multi-GPU TSQR: host-side plumbing (one process per GPU).
+
+The math runs in libcaqr.so: ``caqr_dist_factor_*`` = local TSQR of the shard,
+``ncclAllGather`` of the n x n local R factors over NVLink, and the same
+deterministic combine tree on every rank (``caqr_combine_*``) -- the
+distributed TSQR the paper cites with the GPUs as the leaves of
+one more tree level.  This module only
+  * decides the contiguous row shards (``shard_rows``),
+  * creates the NCCL communicator inside libcaqr from a ``ncclUniqueId`` that
+    rank 0 makes and torch.distributed broadcasts (``DistTSQR``),
+  * offers ``allgather_r`` -- the same exchange through torch.distributed
+    (any backend, incl. gloo on CPU), used to test the exchange order and by
+    callers that already hold a torch process group.
+"""
+from __future__ import annotations
+
+import ctypes
+from typing import Tuple
+
+
+def shard_rows(m: int, world: int, rank: int) -> Tuple[int, int]:
+    """Contiguous row shard of rank `rank`: (first_row, rows).  Even split,
+    remainder to the last rank."""
+    if world < 1 or not 0 <= rank < world:
+        raise ValueError("bad world/rank")
+    base = m // world
+    start = rank * base
+    rows = base if rank < world - 1 else m - start
+    return start, rows
+
+
+def check_shards(m: int, n: int, world: int) -> None:
+    """Every shard must hold at least n rows (each local R is n x n)."""
+    for r in range(world):
+        _, rows = shard_rows(m, world, r)
+        if rows < n:
+            raise ValueError(f"rank {r} would get {rows} < n = {n} rows; use fewer ranks")
+
+
+def allgather_r(R_local, group=None):
+    """Stack every rank's n x n R (rank order) into a (world*n) x n tensor via
+    torch.distributed.all_gather (works for gloo CPU tensors and NCCL CUDA
+    tensors).  Returns the stacked tensor (row-major torch layout)."""
+    import torch
+    import torch.distributed as dist
+
+    world = dist.get_world_size(group)
+    parts = [torch.empty_like(R_local) for _ in range(world)]
+    dist.all_gather(parts, R_local.contiguous(), group=group)
+    return torch.cat(parts, dim=0)
+
+
+class DistTSQR:
+    """NCCL communicator owned by libcaqr (caqr_dist_create) for the ranks of a
+    torch.distributed group; `factor` runs caqr_dist_factor_* on a local shard."""
+
+    def __init__(self, group=None):
+        import torch.distributed as dist
+
+        from . import caqr
+
+        self.caqr = caqr
+        self.L = caqr.lib()
+        self.world = dist.get_world_size(group)
+        self.rank = dist.get_rank(group)
+        uid = (ctypes.c_char * 128)()
+        if self.rank == 0:
+            caqr._check("caqr_dist_unique_id", self.L.caqr_dist_unique_id(uid))
+        obj = [bytes(uid)]
+        dist.broadcast_object_list(obj, src=dist.get_global_rank(group, 0) if group is not None else 0,
+                                   group=group)
+        uid = (ctypes.c_char * 128).from_buffer_copy(obj[0])
+        h = ctypes.c_void_p()
+        caqr._check("caqr_dist_create", self.L.caqr_dist_create(ctypes.byref(h), self.world, self.rank, uid))
+        self.handle = h
+
+    def factor(self, A_local, opts=None, stream=None):
+        """Factor the local column-major shard in place; returns (R, ws, gather,
+        cws): the global R (identical bits on every rank), the local workspace,
+        the combine's stacked tree vectors and its workspace."""
+        import torch
+
+        c = self.caqr
+        code, suf = c._dtype_code(A_local)
+        m, n = A_local.shape
+        pa, lda = c._colmajor(A_local, "A")
+        R = c.colmajor_empty(n, n, A_local.dtype, A_local.device)
+        ws = torch.empty(max(c.caqr_workspace_bytes(m, n, code, opts), 1), dtype=torch.uint8,
+                         device=A_local.device)
+        gather = c.colmajor_empty(self.world * n, n, A_local.dtype, A_local.device)
+        cws = torch.empty(c.caqr_combine_workspace_bytes(self.world, n, code), dtype=torch.uint8,
+                          device=A_local.device)
+        info = getattr(self.L, f"caqr_dist_factor_{suf}")(
+            self.handle, m, n, pa, lda, R.data_ptr(), n, ws.data_ptr(), ws.numel(), gather.data_ptr(),
+            cws.data_ptr(), cws.numel(), c._optp(opts), c._stream(stream))
+        c._check(f"caqr_dist_factor_{suf}", info)
+        return R, ws, gather, cws
+
+    def close(self):
+        if getattr(self, "handle", None) is not None:
+            self.L.caqr_dist_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):  # pragma: no cover
+        try:
+            self.close()
+        except Exception:
+            pass

@@ -253,3 +253,34 @@ def test_errors_raise(caqr):
         caqr.caqr_factor(A, opts=caqr.Opts(48, 0))
     with pytest.raises(ValueError):
         caqr.caqr_factor(torch.zeros(10, 4, device="cuda"))  # row-major
+
+
+def test_dist_single_rank_nccl(caqr):
+    """caqr_dist_* through a real NCCL communicator with one rank (the only
+    configuration one GPU allows): local TSQR + all-gather + combine must give
+    exactly the single-GPU R."""
+    import os
+    import socket
+
+    import torch.distributed as dist
+
+    from paper_conf_ipps_andersonbdk11_b200 import dist as cdist
+
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        A = workloads.gaussian(20000, 96, seed=8)
+        R_ref, _, _, _ = gpu_qr(caqr, A, want_q=False)
+        d = cdist.DistTSQR()
+        Ad = to_dev(caqr, A)
+        R, ws, gather, cws = d.factor(Ad)
+        torch.cuda.synchronize()
+        assert np.array_equal(R.cpu().numpy().astype(np.float64), R_ref)
+        d.close()
+    finally:
+        dist.destroy_process_group()
