@@ -61,9 +61,11 @@ enum { CAQR_F32 = 0, CAQR_F64 = 1 };
 enum { CAQR_OK = 0, CAQR_ERR_CUDA = 1, CAQR_ERR_NCCL = 2, CAQR_ERR_UNSUPPORTED = 3 };
 
 /* Plan options; a field <= 0 means "default".
- *   leaf_rows  b: rows per TSQR leaf (P:L633 / P:L822-823 used 64 and 128 on
+ *   leaf_rows  b: rows per TSQR tile (P:L633 / P:L822-823 used 64 and 128 on
  *              Fermi; here a multiple of 32, b >= the panel-group width,
- *              b <= 256).  Default 256.
+ *              b <= 256).  Default 224 (256 for groups wider than 224).
+ *              Consecutive tiles form chains (flat trees) of K = ceil(L/296)
+ *              tiles; the chains' R factors are reduced by a binary tree.
  *   panel_cols nb: CAQR panel-group width (one TSQR per group).
  *              Default: n if n <= 256 (one whole-width TSQR), else 64. */
 typedef struct caqr_opts {
@@ -203,8 +205,8 @@ const char *caqr_kernel_name(int id);
 int caqr_debug_profile_read(unsigned long long out[16]);
 
 /* Plan introspection (host only; for tests and the bench's roofline bookkeeping).
- * Fills out[0..7] = {leaf_rows, panel_cols, groups, leaves(group 0),
- * tree_levels(group 0), panels(group 0), kernel_launches(factor), 0}.
+ * Fills out[0..7] = {leaf_rows, panel_cols, groups, tiles(group 0),
+ * tree_levels(group 0), panels(group 0), kernel_launches(factor), chains(group 0)}.
  * Returns 0 or a negative info. */
 int caqr_plan_info(int64_t m, int64_t n, int dtype, const caqr_opts *opts, int64_t out[8]);
 

@@ -183,7 +183,7 @@ def caqr_workspace_bytes(m: int, n: int, dtype: int = CAQR_F32, opts: Optional[O
 def caqr_plan_info(m: int, n: int, dtype: int = CAQR_F32, opts: Optional[Opts] = None) -> dict:
     out = (ctypes.c_int64 * 8)()
     _check("caqr_plan_info", lib().caqr_plan_info(m, n, dtype, _optp(opts), out))
-    keys = ["leaf_rows", "panel_cols", "groups", "leaves", "tree_levels", "panels", "launches"]
+    keys = ["leaf_rows", "panel_cols", "groups", "leaves", "tree_levels", "panels", "launches", "chains"]
     return {k: int(out[i]) for i, k in enumerate(keys)}
 
 

@@ -54,8 +54,10 @@ struct TraceScope {  // records a start event now and a stop event at destructio
     }
 };
 
-constexpr int64_t kMaxGroup = 256;  // widest single TSQR panel group
-constexpr int64_t kMaxLeaf = 256;   // tallest leaf the v1 kernels stage in shared memory
+constexpr int64_t kMaxGroup = 256;    // widest single TSQR panel group
+constexpr int64_t kMaxLeaf = 256;     // tallest tile the kernels stage in shared memory
+constexpr int64_t kFusedLeaf = 224;   // default tile height: [32 R rows; tile] fits 256 rows
+constexpr int64_t kChainTarget = 296; // chains per group (2 per B200 SM; device-independent constant)
 
 struct Plan {
     int64_t m = 0, n = 0;
@@ -76,7 +78,7 @@ static int make_plan(int64_t m, int64_t n, int dtype, const caqr_opts* o, int op
     int64_t nb = (o && o->panel_cols > 0) ? o->panel_cols : (n <= kMaxGroup ? n : 64);
     if (nb > kMaxGroup) return -opt_pos;
     nb = std::max<int64_t>(1, std::min(nb, std::max<int64_t>(n, 1)));
-    int64_t b = (o && o->leaf_rows > 0) ? o->leaf_rows : kMaxLeaf;
+    int64_t b = (o && o->leaf_rows > 0) ? o->leaf_rows : (nb <= kFusedLeaf ? kFusedLeaf : kMaxLeaf);
     if (b % 32 != 0 || b > kMaxLeaf) return -opt_pos;
     b = std::max(b, round_up(nb, 32));
     if (b > kMaxLeaf) return -opt_pos;
@@ -96,6 +98,9 @@ static Geom group_geom(const Plan& pl, int64_t g, int64_t lda) {
     G.npan = (int32_t)ceil_div(G.ncols, kPW);
     G.b = pl.b;
     G.L = std::max<int64_t>(1, ceil_div(G.mrows, pl.b));
+    G.K = ceil_div(G.L, kChainTarget);
+    G.P = ceil_div(G.L, G.K);
+    G.bm = G.K * G.b;
     return G;
 }
 
@@ -132,6 +137,7 @@ static size_t plan_ws_bytes(const Plan& pl) {
 // must fit its 256-row register layout: leaves (b rows) and merges (2 wp + 32 p).
 static bool fused_ok(const Geom& G) {
     if (G.b > kFusedMaxRows) return false;
+    if (G.K > 1 && 32 + G.b > kFusedMaxRows) return false;  // [chain R; tile] nodes
     for (int p = 0; p < G.npan; ++p) {
         const int wp = std::min<int>(kPW, G.ncols - 32 * p);
         if (2 * wp + 32 * p > kFusedMaxRows) return false;
@@ -152,26 +158,28 @@ static int num_sms() {
 // ---- launch helpers ---------------------------------------------------------
 
 // Host replica of node_rows()'s gathered-row count (trace bookkeeping only).
-static int64_t node_rg(const Geom& G, int level, int64_t node, int p, int wp) {
+static int64_t node_rg(const Geom& G, int level, int64_t node, int p, int wp, int kt) {
     if (level < 0) {
-        const int64_t h = std::min(G.b, G.mrows - node * G.b);
-        return std::max<int64_t>(0, h - 32 * p);
+        const int64_t t = node * G.K + kt;
+        if (t >= G.L) return 0;
+        const int64_t h = std::min(G.b, G.mrows - t * G.b);
+        return kt == 0 ? std::max<int64_t>(0, h - 32 * p) : wp + h;
     }
     const int64_t a = node << (level + 1), bb = a + (int64_t(1) << level);
-    const int64_t hb = std::min(G.b, G.mrows - bb * G.b);
+    const int64_t hb = std::min(G.b, G.mrows - bb * G.bm);
     return wp + std::min<int64_t>(32 * p + wp, hb);
 }
 // Algorithmic work of one launch: Householder QR of each node's gathered
 // RG x wp panel (LAPACK count) / the two GEMMs of the blocked update
 // (4 RG wp ccount); bytes = the panel / C block read and written once (+ V).
-static void trace_counts(const Geom& G, int level, int p, int64_t nodes, bool update,
+static void trace_counts(const Geom& G, int level, int p, int kt, int64_t nodes, bool update,
                          int64_t ccount, size_t es, double* fl, double* by) {
     *fl = 0;
     *by = 0;
     if (!g_trace.on) return;
     const int wp = std::min<int>(kPW, G.ncols - 32 * p);
     for (int64_t nd = 0; nd < nodes; ++nd) {
-        const double rg = (double)node_rg(G, level, nd, p, wp);
+        const double rg = (double)node_rg(G, level, nd, p, wp, kt);
         const double k = std::min<double>(rg, wp);
         if (!update) {
             *fl += 2.0 * rg * wp * k - 2.0 / 3.0 * k * k * k;
@@ -215,18 +223,19 @@ static cudaError_t allow_smem(K kernel, size_t bytes) {
 }
 
 template <typename T>
-static int launch_factor(const Geom& G, T* A, T* Tws, int level, int p, int64_t nodes,
+static int launch_factor(const Geom& G, T* A, T* Tws, int level, int p, int kt, int64_t nodes,
                          cudaStream_t s) {
     if (nodes <= 0) return 0;
     const int wp = std::min<int>(kPW, G.ncols - 32 * p);
-    const int rgmax = level < 0 ? (int)std::min<int64_t>(G.b, G.mrows) : 2 * wp + 32 * p;
+    const int rgmax = level < 0 ? (kt == 0 ? (int)std::min<int64_t>(G.b, G.mrows) : wp + (int)G.b)
+                                : 2 * wp + 32 * p;
     const size_t smem = panel_factor_smem<T>(wp, rgmax);
     cudaError_t e = allow_smem(panel_factor_kernel<T>, smem);
     double fl, by;
-    trace_counts(G, level, p, nodes, false, 0, sizeof(T), &fl, &by);
+    trace_counts(G, level, p, kt, nodes, false, 0, sizeof(T), &fl, &by);
     TraceScope ts(K_PANEL_FACTOR, fl, by, s);
     if (e == cudaSuccess) {
-        panel_factor_kernel<T><<<dim3((unsigned)nodes), kThreads, smem, s>>>(G, A, Tws, level, p);
+        panel_factor_kernel<T><<<dim3((unsigned)nodes), kThreads, smem, s>>>(G, A, Tws, level, p, kt);
         e = cudaGetLastError();
     }
     if (e != cudaSuccess) {
@@ -237,20 +246,21 @@ static int launch_factor(const Geom& G, T* A, T* Tws, int level, int p, int64_t 
 }
 
 template <typename T>
-static int launch_update(const Geom& G, const T* A, const T* Tws, int level, int p, int64_t nodes,
-                         T* C, int64_t ldc, int64_t cfirst, int64_t ccount, int trans,
+static int launch_update(const Geom& G, const T* A, const T* Tws, int level, int p, int kt,
+                         int64_t nodes, T* C, int64_t ldc, int64_t cfirst, int64_t ccount, int trans,
                          cudaStream_t s) {
     if (nodes <= 0 || ccount <= 0) return 0;
     const int wp = std::min<int>(kPW, G.ncols - 32 * p);
-    const int rgmax = level < 0 ? (int)std::min<int64_t>(G.b, G.mrows) : 2 * wp + 32 * p;
+    const int rgmax = level < 0 ? (kt == 0 ? (int)std::min<int64_t>(G.b, G.mrows) : wp + (int)G.b)
+                                : 2 * wp + 32 * p;
     const size_t smem = panel_update_smem<T>(rgmax);
     cudaError_t e = allow_smem(panel_update_kernel<T>, smem);
     double fl, by;
-    trace_counts(G, level, p, nodes, true, ccount, sizeof(T), &fl, &by);
+    trace_counts(G, level, p, kt, nodes, true, ccount, sizeof(T), &fl, &by);
     TraceScope ts(K_PANEL_UPDATE, fl, by, s);
     if (e == cudaSuccess) {
         dim3 grid((unsigned)nodes, (unsigned)ceil_div(ccount, 32));
-        panel_update_kernel<T><<<grid, kThreads, smem, s>>>(G, A, Tws, level, p, C, ldc, cfirst,
+        panel_update_kernel<T><<<grid, kThreads, smem, s>>>(G, A, Tws, level, p, kt, C, ldc, cfirst,
                                                             ccount, trans);
         e = cudaGetLastError();
     }
@@ -278,9 +288,9 @@ static unsigned long long* prof_buffer() {
 // The whole TSQR of a group (leaves + every tree level) in one persistent launch.
 template <typename T>
 static int launch_fused(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, cudaStream_t s) {
-    const int nl = tree_levels(G.L);
-    int64_t total = do_leaves ? G.L : 0;
-    for (int lv = 0; lv < nl; ++lv) total += merges_at(G.L, lv);
+    const int nl = tree_levels(G.P);
+    int64_t total = do_leaves ? G.P : 0;
+    for (int lv = 0; lv < nl; ++lv) total += merges_at(G.P, lv);
     if (total <= 0) return 0;
     cudaError_t e = cudaMemsetAsync(sync, 0, group_sync_bytes(G), s);
     const size_t smem = fused_smem_bytes<T>();
@@ -294,7 +304,7 @@ static int launch_fused(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, 
         if (g_trace.on) {
             const double mr = (double)G.mrows, nc = (double)G.ncols;
             fl = do_leaves ? 2.0 * mr * nc * nc - 2.0 / 3.0 * nc * nc * nc
-                           : (double)(G.L - 1) * 2.0 / 3.0 * nc * nc * nc;
+                           : (double)(G.P - 1) * 2.0 / 3.0 * nc * nc * nc;
             by = 2.0 * mr * nc * sizeof(T);
         }
         TraceScope ts(K_TSQR_FUSED, fl, by, s);
@@ -309,13 +319,11 @@ static int launch_fused(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, 
     return 0;
 }
 
+// CAQR_FUSED=0 forces the split (one launch per level and panel) path; read
+// on every call so tests can compare both paths in one process.
 static inline int fused_policy() {
-    static int v = -1;
-    if (v < 0) {
-        const char* e = getenv("CAQR_FUSED");
-        v = (e && e[0] == '0') ? 0 : 1;
-    }
-    return v;
+    const char* e = getenv("CAQR_FUSED");
+    return (e && e[0] == '0') ? 0 : 1;
 }
 
 // TSQR of one panel group (Fig. 4 minus the trailing update): every leaf's
@@ -325,20 +333,21 @@ static int factor_group(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, 
     if (fused_policy() && fused_ok(G)) return launch_fused<T>(G, A, Tws, sync, do_leaves, s);
     int rc = 0;
     if (do_leaves) {
-        for (int p = 0; p < G.npan && !rc; ++p) {
-            rc = launch_factor<T>(G, A, Tws, -1, p, G.L, s);
-            if (!rc && p + 1 < G.npan)
-                rc = launch_update<T>(G, A, Tws, -1, p, G.L, A, G.lda, G.col0 + 32 * (p + 1),
-                                      G.ncols - 32 * (p + 1), 1, s);
-        }
+        for (int kt = 0; kt < G.K && !rc; ++kt)
+            for (int p = 0; p < G.npan && !rc; ++p) {
+                rc = launch_factor<T>(G, A, Tws, -1, p, kt, G.P, s);
+                if (!rc && p + 1 < G.npan)
+                    rc = launch_update<T>(G, A, Tws, -1, p, kt, G.P, A, G.lda, G.col0 + 32 * (p + 1),
+                                          G.ncols - 32 * (p + 1), 1, s);
+            }
     }
-    const int nl = tree_levels(G.L);
+    const int nl = tree_levels(G.P);
     for (int lv = 0; lv < nl && !rc; ++lv) {
-        const int64_t nm = merges_at(G.L, lv);
+        const int64_t nm = merges_at(G.P, lv);
         for (int p = 0; p < G.npan && !rc; ++p) {
-            rc = launch_factor<T>(G, A, Tws, lv, p, nm, s);
+            rc = launch_factor<T>(G, A, Tws, lv, p, 0, nm, s);
             if (!rc && p + 1 < G.npan)
-                rc = launch_update<T>(G, A, Tws, lv, p, nm, A, G.lda, G.col0 + 32 * (p + 1),
+                rc = launch_update<T>(G, A, Tws, lv, p, 0, nm, A, G.lda, G.col0 + 32 * (p + 1),
                                       G.ncols - 32 * (p + 1), 1, s);
         }
     }
@@ -352,23 +361,25 @@ template <typename T>
 static int apply_group(const Geom& G, const T* A, const T* Tws, bool do_leaves, T* C,
                        int64_t ldc, int64_t cfirst, int64_t ccount, int trans, cudaStream_t s) {
     int rc = 0;
-    const int nl = tree_levels(G.L);
+    const int nl = tree_levels(G.P);
     if (trans) {
         if (do_leaves)
-            for (int p = 0; p < G.npan && !rc; ++p)
-                rc = launch_update<T>(G, A, Tws, -1, p, G.L, C, ldc, cfirst, ccount, 1, s);
+            for (int kt = 0; kt < G.K && !rc; ++kt)
+                for (int p = 0; p < G.npan && !rc; ++p)
+                    rc = launch_update<T>(G, A, Tws, -1, p, kt, G.P, C, ldc, cfirst, ccount, 1, s);
         for (int lv = 0; lv < nl && !rc; ++lv)
             for (int p = 0; p < G.npan && !rc; ++p)
-                rc = launch_update<T>(G, A, Tws, lv, p, merges_at(G.L, lv), C, ldc, cfirst, ccount,
+                rc = launch_update<T>(G, A, Tws, lv, p, 0, merges_at(G.P, lv), C, ldc, cfirst, ccount,
                                       1, s);
     } else {
         for (int lv = nl - 1; lv >= 0 && !rc; --lv)
             for (int p = G.npan - 1; p >= 0 && !rc; --p)
-                rc = launch_update<T>(G, A, Tws, lv, p, merges_at(G.L, lv), C, ldc, cfirst, ccount,
+                rc = launch_update<T>(G, A, Tws, lv, p, 0, merges_at(G.P, lv), C, ldc, cfirst, ccount,
                                       0, s);
         if (do_leaves)
-            for (int p = G.npan - 1; p >= 0 && !rc; --p)
-                rc = launch_update<T>(G, A, Tws, -1, p, G.L, C, ldc, cfirst, ccount, 0, s);
+            for (int kt = (int)G.K - 1; kt >= 0 && !rc; --kt)
+                for (int p = G.npan - 1; p >= 0 && !rc; --p)
+                    rc = launch_update<T>(G, A, Tws, -1, p, kt, G.P, C, ldc, cfirst, ccount, 0, s);
     }
     return rc;
 }
@@ -493,6 +504,9 @@ static Geom combine_geom(int P, int64_t n, int64_t ld) {
     G.npan = (int32_t)ceil_div(n, kPW);
     G.b = n;
     G.L = P;
+    G.K = 1;
+    G.P = P;
+    G.bm = n;
     return G;
 }
 
@@ -687,14 +701,18 @@ int caqr_plan_info(int64_t m, int64_t n, int dtype, const caqr_opts* opts, int64
     if (pl.ngroups == 0) return 0;
     const Geom G = group_geom(pl, 0, m);
     out[3] = G.L;
-    out[4] = tree_levels(G.L);
+    out[4] = tree_levels(G.P);
     out[5] = G.npan;
+    out[7] = G.P;
     int64_t launches = 1;  // extract_r
     for (int64_t g = 0; g < pl.ngroups; ++g) {
         const Geom Gg = group_geom(pl, g, m);
-        const int nl = tree_levels(Gg.L);
-        launches += (int64_t)(nl + 1) * (2 * Gg.npan - 1);
-        if (Gg.col0 + Gg.ncols < n) launches += (int64_t)(nl + 1) * Gg.npan;
+        const int nl = tree_levels(Gg.P);
+        if (fused_ok(Gg))
+            launches += 1;
+        else
+            launches += (int64_t)(nl + Gg.K) * (2 * Gg.npan - 1);
+        if (Gg.col0 + Gg.ncols < n) launches += (int64_t)(nl + Gg.K) * Gg.npan;
     }
     out[6] = launches;
     return 0;

@@ -703,11 +703,11 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
     __shared__ int s_task;
     int* ticket = sync;
     int* flags = sync + 32;  // [L][npan]
-    const int64_t leaf_tasks = do_leaves ? g.L : 0;
+    const int64_t leaf_tasks = do_leaves ? g.P : 0;  // one task per chain of K tiles
     int64_t total = leaf_tasks;
     for (int l = 0; l < nlevels; ++l) {
         const int64_t h = int64_t(1) << l;
-        total += (g.L - 1 >= h) ? (g.L - 1 - h) / (2 * h) + 1 : 0;
+        total += (g.P - 1 >= h) ? (g.P - 1 - h) / (2 * h) + 1 : 0;
     }
     // optional phase profile (diagnostics; prof == nullptr in normal use)
     // (accumulators live in shared memory: no registers taken from the math)
@@ -735,7 +735,7 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
             level = 0;
             for (;;) {
                 const int64_t h = int64_t(1) << level;
-                const int64_t nm = (g.L - 1 >= h) ? (g.L - 1 - h) / (2 * h) + 1 : 0;
+                const int64_t nm = (g.P - 1 >= h) ? (g.P - 1 - h) / (2 * h) + 1 : 0;
                 if (node < nm) break;
                 node -= nm;
                 ++level;
@@ -748,13 +748,16 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
         } else {
             slot_a = node << (level + 1);
             slot_b = slot_a + (int64_t(1) << level);
-            ver_a = expected_version(slot_a, level, g.L, do_leaves);
-            ver_b = expected_version(slot_b, level, g.L, do_leaves);
+            ver_a = expected_version(slot_a, level, g.P, do_leaves);
+            ver_b = expected_version(slot_b, level, g.P, do_leaves);
         }
         const int my_ver = level + 2;
+        // a chain walks its tiles in order; a merge is one "tile"
+        const int64_t ntile = level < 0 ? min(g.K, g.L - node * g.K) : 1;
+        for (int kt = 0; kt < ntile; ++kt)
         for (int p = 0; p < g.npan; ++p) {
             const int wp = min(kPW, g.ncols - 32 * p);
-            if (level >= 0 && threadIdx.x == 0) {
+            if (level >= 0 && threadIdx.x == 0) {  // children's panel p must be final
                 const int* fa = flags + slot_a * g.npan + p;
                 const int* fb = flags + slot_b * g.npan + p;
                 while (ld_acquire(fa) < ver_a) __nanosleep(64);
@@ -763,7 +766,7 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
             __syncthreads();
             CAQR_PROF(1);
             if (prof && threadIdx.x == 0) pacc[level < 0 ? 10 : 11] += 1;
-            const NodeRows nr = node_rows(g, level, node, p, wp);
+            const NodeRows nr = node_rows(g, level, node, p, wp, kt);
             const int RG = nr.n0 + nr.n1;
             const int R32 = (RG + 31) & ~31;
             const int64_t c0 = g.col0 + 32 * p;
@@ -783,16 +786,8 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
                         const bool in = r < RG;
                         const T val = pc[padr<T>(r)];
                         if (in && panel_entry_stored(nr, r, jj, p)) col[gathered_row(nr, r)] = val;
-                        // V form in place: unit head, zeros above, merge masks
-                        T v = T(0);
-                        if (in) {
-                            if (!nr.merge)
-                                v = r > jj ? val : (r == jj ? T(1) : T(0));
-                            else if (r < nr.n0)
-                                v = (r == jj) ? T(1) : T(0);
-                            else
-                                v = (r - nr.n0) <= 32 * p + jj ? val : T(0);
-                        }
+                        // V form in place: unit head, zeros above, structure masks
+                        const T v = in ? v_entry<T>(nr, r, jj, p, val) : T(0);
                         pc[padr<T>(r)] = v;
                     }
                 }
@@ -829,7 +824,8 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
             // ---- publish ----------------------------------------------------------
             __threadfence();
             __syncthreads();
-            if (threadIdx.x == 0) st_release(flags + slot_a * g.npan + p, level < 0 ? 1 : my_ver);
+            if (threadIdx.x == 0 && kt == ntile - 1)  // the slot's R rows of panel p are final
+                st_release(flags + slot_a * g.npan + p, level < 0 ? 1 : my_ver);
             CAQR_PROF(9);
         }
     }

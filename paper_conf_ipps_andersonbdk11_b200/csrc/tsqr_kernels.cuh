@@ -37,47 +37,67 @@ constexpr int kTS = 36;        // stride of 32x32 scratch tiles (16-byte aligned
 
 // Geometry of one TSQR panel group (a column panel of width ncols <= 256 that
 // starts at row0 = col0 of A; the grid redrawn "nb rows lower").
+// Rows are cut into L tiles of b rows (the last one ragged).  Consecutive
+// tiles form chains of K tiles (a flat tree, "any tree shape" P:L339-341): the
+// first tile of a chain is a leaf QR, each later tile a structured QR of
+// [chain R; tile].  The P chain R factors are reduced by a binary tree.
 struct Geom {
     int64_t lda;
     int64_t row0;   // first row of the group
     int64_t mrows;  // rows of the group (m - row0)
     int64_t col0;   // first column of the group
-    int64_t b;      // leaf height
-    int64_t L;      // number of leaves
+    int64_t b;      // tile (leaf) height
+    int64_t L;      // number of tiles
+    int64_t K;      // tiles per chain
+    int64_t P;      // chains = leaves of the binary tree
+    int64_t bm;     // rows per chain (K * b): stride of the tree's R slots
     int32_t ncols;  // group width
     int32_t npan;   // ceil(ncols / 32)
 };
 
-// The gathered rows of node `node` at tree `level` (-1 = leaves) for panel p.
+// The gathered rows of one node for panel p.  level < 0: tile kt of chain
+// `node` (kt == 0: leaf); level >= 0: merge `node` of that tree level.
 struct NodeRows {
-    int64_t r0, r1;  // first absolute row of segment 0 / segment 1
-    int32_t n0, n1;  // rows in segment 0 / 1
-    int32_t merge;   // 0 = leaf, 1 = merge of two R factors
-    int64_t tblk;    // index of this (node, panel)'s 32x32 T block in the workspace
+    int64_t r0, r1;      // first absolute row of segment 0 / segment 1
+    int32_t n0, n1;      // rows in segment 0 / 1
+    int32_t seg0_tri;    // 1: segment 0 is an R slot (heads on its diagonal, v = e_j there)
+    int32_t seg1_upper;  // 1: segment 1 is an upper-triangular R slot (merge); 0: dense
+    int64_t tblk;        // index of this (node, panel)'s 32x32 T block in the workspace
 };
 
-__device__ __forceinline__ NodeRows node_rows(const Geom& g, int level, int64_t node, int p,
-                                              int wp) {
+__device__ __forceinline__ NodeRows node_rows(const Geom& g, int level, int64_t node, int p, int wp,
+                                              int kt) {
     NodeRows nr;
     if (level < 0) {
-        const int64_t s = g.row0 + node * g.b;
-        const int64_t h = min(g.b, g.mrows - node * g.b);
-        nr.r0 = s + 32 * p;
-        nr.n0 = (int32_t)(h - 32 * p > 0 ? h - 32 * p : 0);
-        nr.r1 = 0;
-        nr.n1 = 0;
-        nr.merge = 0;
-        nr.tblk = node * g.npan + p;
+        const int64_t t = node * g.K + kt;  // tile index
+        const int64_t s = g.row0 + t * g.b;
+        const int64_t h = t < g.L ? min(g.b, g.mrows - t * g.b) : 0;
+        nr.tblk = t * g.npan + p;
+        nr.seg1_upper = 0;
+        if (kt == 0) {  // leaf
+            nr.r0 = s + 32 * p;
+            nr.n0 = (int32_t)(h - 32 * p > 0 ? h - 32 * p : 0);
+            nr.r1 = 0;
+            nr.n1 = 0;
+            nr.seg0_tri = 0;
+        } else {  // [chain R; tile]
+            nr.r0 = g.row0 + node * g.bm + 32 * p;
+            nr.n0 = h > 0 ? wp : 0;
+            nr.r1 = s;
+            nr.n1 = (int32_t)h;
+            nr.seg0_tri = 1;
+        }
     } else {
         const int64_t a = node << (level + 1);
         const int64_t bb = a + (int64_t(1) << level);
-        const int64_t hb = min(g.b, g.mrows - bb * g.b);
-        nr.r0 = g.row0 + a * g.b + 32 * p;
+        const int64_t hb = min(g.b, g.mrows - bb * g.bm);
+        nr.r0 = g.row0 + a * g.bm + 32 * p;
         nr.n0 = wp;
-        nr.r1 = g.row0 + bb * g.b;
+        nr.r1 = g.row0 + bb * g.bm;
         nr.n1 = (int32_t)(32 * p + wp < hb ? 32 * p + wp : hb);
-        nr.merge = 1;
-        nr.tblk = (g.L + bb) * g.npan + p;
+        nr.seg0_tri = 1;
+        nr.seg1_upper = 1;
+        nr.tblk = (g.L + bb * g.K) * g.npan + p;
     }
     return nr;
 }
@@ -88,14 +108,25 @@ __device__ __forceinline__ int64_t gathered_row(const NodeRows& nr, int r) {
 }
 
 // Is entry (gathered row r, panel column jj) of the panel stored in A for this
-// node?  Leaves: every entry (R on/above the diagonal, v below).  Merges: R_a's
-// rows hold R on and above the diagonal only (below it sit leaf vectors);
-// R_b's rows hold an upper-triangular R (factor input) / V_2 (tree vectors)
-// only -- local row i <= 32p + jj.
+// node?  Leaves and dense tiles: every entry (R on/above the diagonal, v
+// below).  An R-slot segment 0 holds R on and above the diagonal only (below it
+// sit leaf vectors); a merge's R_b segment holds an upper-triangular R (factor
+// input) / V_2 (tree vectors) only -- local row i <= 32p + jj.
 __device__ __forceinline__ bool panel_entry_stored(const NodeRows& nr, int r, int jj, int p) {
-    if (!nr.merge) return true;
-    if (r < nr.n0) return r <= jj;
-    return (r - nr.n0) <= 32 * p + jj;
+    if (r < nr.n0) return !nr.seg0_tri || r <= jj;
+    return !nr.seg1_upper || (r - nr.n0) <= 32 * p + jj;
+}
+
+// Householder vector entry (gathered row r, panel column jj) given the stored
+// value: unit head, zeros above it, the structure's zeros.
+template <typename T>
+__device__ __forceinline__ T v_entry(const NodeRows& nr, int r, int jj, int p, T stored) {
+    if (r < nr.n0) {
+        if (nr.seg0_tri) return r == jj ? T(1) : T(0);
+        return r > jj ? stored : (r == jj ? T(1) : T(0));
+    }
+    if (nr.seg1_upper) return (r - nr.n0) <= 32 * p + jj ? stored : T(0);
+    return stored;
 }
 
 template <typename T>
@@ -150,11 +181,11 @@ __device__ __forceinline__ void make_reflector(T* P, int RGP, int RG, int j, T* 
 // ---------------------------------------------------------------------------
 template <typename T>
 __global__ void __launch_bounds__(kThreads)
-panel_factor_kernel(Geom g, T* A, T* __restrict__ Tws, int level, int p) {
+panel_factor_kernel(Geom g, T* A, T* __restrict__ Tws, int level, int p, int kt) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int wp = min(kPW, g.ncols - 32 * p);
-    const NodeRows nr = node_rows(g, level, blockIdx.x, p, wp);
+    const NodeRows nr = node_rows(g, level, blockIdx.x, p, wp, kt);
     const int RG = nr.n0 + nr.n1;
     const int RGP = smem_col_stride<T>(RG);
     T* P = reinterpret_cast<T*>(smem_raw);
@@ -275,14 +306,14 @@ __device__ __forceinline__ T vget(const double2& v, int i) {
 
 template <typename T>
 __global__ void __launch_bounds__(kThreads)
-panel_update_kernel(Geom g, const T* A, const T* __restrict__ Tws, int level, int p, T* C,
+panel_update_kernel(Geom g, const T* A, const T* __restrict__ Tws, int level, int p, int kt, T* C,
                     int64_t ldc, int64_t cfirst, int64_t ccount, int trans) {
     using V4 = typename Vec4<T>::type;
     constexpr int VN = Vec4<T>::n;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int wp = min(kPW, g.ncols - 32 * p);
-    const NodeRows nr = node_rows(g, level, blockIdx.x, p, wp);
+    const NodeRows nr = node_rows(g, level, blockIdx.x, p, wp, kt);
     const int RG = nr.n0 + nr.n1;
     if (RG == 0) return;
     const int R32 = (RG + 31) & ~31;
@@ -306,13 +337,9 @@ panel_update_kernel(Geom g, const T* A, const T* __restrict__ Tws, int level, in
             T v = T(0), cv = T(0);
             if (r < RG) {
                 if (jj < wp) {
-                    if (!nr.merge) {
-                        v = r > jj ? acol[gathered_row(nr, r)] : (r == jj ? T(1) : T(0));
-                    } else if (r < nr.n0) {
-                        v = (r == jj) ? T(1) : T(0);
-                    } else {
-                        v = (r - nr.n0) <= 32 * p + jj ? acol[nr.r1 + (r - nr.n0)] : T(0);
-                    }
+                    const bool st = panel_entry_stored(nr, r, jj, p) && (r >= nr.n0 || !nr.seg0_tri) &&
+                                    !(r < nr.n0 && r <= jj);
+                    v = v_entry<T>(nr, r, jj, p, st ? acol[gathered_row(nr, r)] : T(0));
                 }
                 if (jj < ncb) cv = ccol[gathered_row(nr, r)];
             }

@@ -39,9 +39,11 @@ def test_workspace_bytes(L):
     # plus the fused kernel's ticket + (slot, panel) flags: (32 + L*npan) ints, 256-B rounded
     def ws(L, npan, es):
         return 2 * L * npan * 1024 * es + -(-(32 + L * npan) * 4 // 256) * 256
-    assert caqr.caqr_workspace_bytes(4096, 16) == ws(16, 1, 4)
-    assert caqr.caqr_workspace_bytes(4096, 16, caqr.CAQR_F64) == ws(16, 1, 8)
-    assert caqr.caqr_workspace_bytes(1_000_000, 192) == ws(3907, 6, 4)
+    # default tile height 224 (n <= 224): 4096 rows -> 19 tiles; 1M rows -> 4465 tiles
+    assert caqr.caqr_workspace_bytes(4096, 16) == ws(19, 1, 4)
+    assert caqr.caqr_workspace_bytes(4096, 16, caqr.CAQR_F64) == ws(19, 1, 8)
+    assert caqr.caqr_workspace_bytes(1_000_000, 192) == ws(4465, 6, 4)
+    assert caqr.caqr_workspace_bytes(4096, 16, 0, caqr.make_opts(leaf_rows=256)) == ws(16, 1, 4)
     assert caqr.caqr_workspace_bytes(10, 11) == 0  # n > m
     assert caqr.caqr_workspace_bytes(-1, 1) == 0
     assert caqr.caqr_workspace_bytes(10, 2, 7) == 0  # bad dtype
@@ -50,8 +52,10 @@ def test_workspace_bytes(L):
 
 def test_plan_info(L):
     p = caqr.caqr_plan_info(1_000_000, 192)
-    assert p["leaf_rows"] == 256 and p["panel_cols"] == 192 and p["groups"] == 1
-    assert p["leaves"] == 3907 and p["tree_levels"] == 12 and p["panels"] == 6
+    assert p["leaf_rows"] == 224 and p["panel_cols"] == 192 and p["groups"] == 1
+    # 4465 tiles in chains of K = ceil(4465/296) = 16 -> 280 chains -> 9 tree levels
+    assert p["leaves"] == 4465 and p["chains"] == 280 and p["tree_levels"] == 9 and p["panels"] == 6
+    assert p["launches"] == 2  # one fused TSQR kernel + extract_r
     p = caqr.caqr_plan_info(8192, 8192)
     assert p["panel_cols"] == 64 and p["groups"] == 128
     p = caqr.caqr_plan_info(4096, 16, 0, caqr.make_opts(leaf_rows=128))

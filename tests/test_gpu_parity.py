@@ -154,10 +154,11 @@ def test_power_of_two_column_scaling_bitwise(caqr):
 def test_zero_row_padding_bitwise(caqr):
     """R([A; 0]) == R(A) bitwise when the padding fills whole leaves: zero
     leaves merge with tau = 0 (reading S2)."""
+    opts = caqr.make_opts(leaf_rows=256)
     A = workloads.gaussian(256 * 5, 40, seed=4)
     Z = np.vstack([A, np.zeros((256 * 3, 40), np.float32)])
-    R, _, _, _ = gpu_qr(caqr, A, want_q=False)
-    Rz, _, _, _ = gpu_qr(caqr, Z, want_q=False)
+    R, _, _, _ = gpu_qr(caqr, A, opts, want_q=False)
+    Rz, _, _, _ = gpu_qr(caqr, Z, opts, want_q=False)
     assert np.array_equal(R, Rz)
 
 
@@ -167,8 +168,9 @@ def test_row_permutation_of_leaves(caqr):
     A = workloads.gaussian(b * 8, 32, seed=6)
     perm = np.random.default_rng(0).permutation(8)
     Ap = np.vstack([A[i * b:(i + 1) * b] for i in perm])
-    R, _, _, _ = gpu_qr(caqr, A, want_q=False)
-    Rp, _, _, _ = gpu_qr(caqr, Ap, want_q=False)
+    opts = caqr.make_opts(leaf_rows=b)
+    R, _, _, _ = gpu_qr(caqr, A, opts, want_q=False)
+    Rp, _, _, _ = gpu_qr(caqr, Ap, opts, want_q=False)
     Rn, Rpn = oracle.normalize_signs(R), oracle.normalize_signs(Rp)
     assert np.linalg.norm(Rn - Rpn) / np.linalg.norm(Rn) <= 1e-5
 
@@ -284,3 +286,29 @@ def test_dist_single_rank_nccl(caqr):
         d.close()
     finally:
         dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("m,n,leaf", [(20000, 24, 32), (40000, 48, 64), (70000, 100, 128), (70000, 192, 224)])
+@pytest.mark.parametrize("path", ["fused", "split"])
+def test_chains(caqr, m, n, leaf, path, monkeypatch):
+    """More tiles than the chain target (296): tiles form flat-tree chains of
+    K > 1 tiles ([chain R; tile] steps), then the binary tree over chains.
+    Both the one-launch dataflow kernel and the split path."""
+    if path == "split":
+        monkeypatch.setenv("CAQR_FUSED", "0")
+    opts = caqr.make_opts(leaf_rows=leaf)
+    info = caqr.caqr_plan_info(m, n, 0, opts)
+    assert info["leaves"] > 296 and info["chains"] < info["leaves"]
+    A = workloads.gaussian(m, n, seed=m + n)
+    check_against_oracle(caqr, A, opts=opts, C_cols=2)
+
+
+def test_fused_and_split_agree(caqr, monkeypatch):
+    """The two execution paths run the same plan: results agree to rounding
+    (different reduction orders inside the panel factorization)."""
+    A = workloads.gaussian(70000, 64, seed=1)
+    opts = caqr.make_opts(leaf_rows=64)
+    R1, _, _, _ = gpu_qr(caqr, A, opts, want_q=False)
+    monkeypatch.setenv("CAQR_FUSED", "0")
+    R2, _, _, _ = gpu_qr(caqr, A, opts, want_q=False)
+    assert np.linalg.norm(R1 - R2) / np.linalg.norm(R1) <= 1e-5
