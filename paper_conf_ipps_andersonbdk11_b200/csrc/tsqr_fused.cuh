@@ -281,6 +281,49 @@ __device__ __forceinline__ void factor_panel_regs(T* P, int RGP, int RG, int wp,
     __syncthreads();
 }
 
+// A group of 256 threads (8 warps) that runs one device routine: the whole
+// CTA in the one-role kernel, or one of the two roles of the look-ahead
+// kernel (named barrier per role).  tid is the group-local thread index.
+struct Grp {
+    int tid;
+    int bar;  // 0: __syncthreads over the CTA; >0: bar.sync bar, 256
+};
+__device__ __forceinline__ void gsync(const Grp& g) {
+    if (g.bar == 0)
+        __syncthreads();
+    else
+        asm volatile("bar.sync %0, 256;" ::"r"(g.bar) : "memory");
+}
+
+// Sum N values across the 32 lanes of a warp; every lane gets all N totals.
+// Measured on B200: a 5-level SHFL butterfly costs ~150 cycles and SHFL issue
+// is ~9 cycles, so N interleaved butterflies (5N shuffles) are throughput-bound
+// (16 values: ~760 cycles).  Transpose through shared memory instead: each lane
+// stores its N partials, lane l sums value l % NP over a group of NP rows, a
+// few shuffles combine the groups, and the totals are broadcast back.
+// `scr` is this warp's private scratch of 32 * (NP + 4) + NP elements.
+template <int N, typename T>
+__device__ __forceinline__ void warp_reduce_many(T (&v)[N], T* scr) {
+    constexpr int NP = N <= 1 ? 1 : N <= 2 ? 2 : N <= 4 ? 4 : N <= 8 ? 8 : N <= 16 ? 16 : 32;
+    constexpr int LD = NP + 4;  // row stride (16-byte aligned rows, spread banks)
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int k = 0; k < NP; ++k) scr[lane * LD + k] = k < N ? v[k] : T(0);
+    __syncwarp();
+    const int k = lane % NP, g = lane / NP;
+    T acc = T(0);
+#pragma unroll
+    for (int r = 0; r < NP; ++r) acc += scr[(g * NP + r) * LD + k];
+#pragma unroll
+    for (int o = NP; o < 32; o <<= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    __syncwarp();
+    if (lane < NP) scr[32 * LD + lane] = acc;
+    __syncwarp();
+#pragma unroll
+    for (int q = 0; q < N; ++q) v[q] = scr[32 * LD + q];
+    __syncwarp();
+}
+
 // ---------------------------------------------------------------------------
 // Panel factorization, 4-column blocks ("WB4").  Warp w owns panel columns
 // 4w..4w+3; lane l holds rows l + 32 i (i < 8) of each of them in registers
@@ -293,10 +336,16 @@ __device__ __forceinline__ void factor_panel_regs(T* P, int RGP, int RG, int wp,
 // tau_s[0..wp) the reflector scalars.
 // ---------------------------------------------------------------------------
 template <typename T>
-__device__ __forceinline__ void factor_panel_wb4(T* P, int RGP, int RG, int wp, T* tau_s, T* Tb) {
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int cb = 4 * warp;
+__device__ __forceinline__ void factor_panel_wb4(const Grp& G, T* P, int RGP, int RG, int wp, T* tau_s, T* Tb,
+                                                 T* scr_all) {
+    const int warp = G.tid >> 5, lane = G.tid & 31;
+    // block blk = 7 - warp: the warp that owns the next block always has the
+    // highest warp id among the warps still applying the current one, so the
+    // scheduler (highest-id-first) favours the critical path
+    const int blk = kWarps - 1 - warp;
+    const int cb = 4 * blk;
     const int nc = max(0, min(4, wp - cb));
+    T* scr = scr_all + warp * (32 * 20 + 16);  // warp-private reduction scratch
     T x[4][8];
 #pragma unroll
     for (int q = 0; q < 4; ++q)
@@ -305,10 +354,10 @@ __device__ __forceinline__ void factor_panel_wb4(T* P, int RGP, int RG, int wp, 
             const int r = lane + 32 * i;
             x[q][i] = (q < nc && r < RG) ? P[(size_t)(cb + q) * RGP + padr<T>(r)] : T(0);
         }
-    __syncthreads();  // all columns are in registers before P gets v's
+    gsync(G);  // all columns are in registers before P gets v's
     const int nblk = (wp + 3) / 4;
     for (int b = 0; b < nblk; ++b) {
-        if (warp == b) {
+        if (blk == b) {
             T tq[4] = {T(0), T(0), T(0), T(0)};
 #pragma unroll
             for (int q = 0; q < 4; ++q) {
@@ -344,16 +393,19 @@ __device__ __forceinline__ void factor_panel_wb4(T* P, int RGP, int RG, int wp, 
                     }
                     if (lane == 0) tau_s[j] = tau;
                     // apply H_j to this warp's later columns (interleaved reductions)
-                    if (tau != T(0)) {
+                    if (tau != T(0) && q + 1 < nc) {
                         T d[4] = {T(0), T(0), T(0), T(0)};
 #pragma unroll
                         for (int q2 = q + 1; q2 < 4; ++q2)
 #pragma unroll
                             for (int i = 0; i < 8; ++i) d[q2] = fma(v[i], x[q2][i], d[q2]);
+                        if (q == 0)
+                            warp_reduce_many<4>(d, scr);
+                        else
 #pragma unroll
-                        for (int o = 16; o > 0; o >>= 1)
+                            for (int o = 16; o > 0; o >>= 1)
 #pragma unroll
-                            for (int q2 = q + 1; q2 < 4; ++q2) d[q2] += __shfl_xor_sync(0xffffffffu, d[q2], o);
+                                for (int q2 = q + 1; q2 < 4; ++q2) d[q2] += __shfl_xor_sync(0xffffffffu, d[q2], o);
 #pragma unroll
                         for (int q2 = q + 1; q2 < 4; ++q2) {
                             const T st = tau * d[q2];
@@ -385,10 +437,7 @@ __device__ __forceinline__ void factor_panel_wb4(T* P, int RGP, int RG, int wp, 
                         for (int i = 0; i < 8; ++i) g = fma(vv[a][i], vv[bb][i], g);
                         gv[e] = g;
                     }
-#pragma unroll
-                for (int o = 16; o > 0; o >>= 1)
-#pragma unroll
-                    for (int k = 0; k < 6; ++k) gv[k] += __shfl_xor_sync(0xffffffffu, gv[k], o);
+                warp_reduce_many<6>(gv, scr);
             }
             if (lane == 0) {
                 // gv index of (a, bb), a < bb: 0:(0,1) 1:(0,2) 2:(0,3) 3:(1,2) 4:(1,3) 5:(2,3)
@@ -412,8 +461,8 @@ __device__ __forceinline__ void factor_panel_wb4(T* P, int RGP, int RG, int wp, 
                     for (int bb = 0; bb < 4; ++bb) Tb[b * 16 + a * 4 + bb] = tm[a][bb];
             }
         }
-        __syncthreads();
-        if (warp > b && nc > 0) {
+        gsync(G);
+        if (blk > b && nc > 0) {
             // X <- X - V_b (T_b^T (V_b^T X)) on this warp's columns
             T vb[4][8];
             const int jb = 4 * b;
@@ -431,12 +480,18 @@ __device__ __forceinline__ void factor_panel_wb4(T* P, int RGP, int RG, int wp, 
                     for (int i = 0; i < 8; ++i) acc = fma(vb[a][i], x[q][i], acc);
                     w[a][q] = acc;
                 }
-#pragma unroll
-            for (int o = 16; o > 0; o >>= 1)
+            {
+                T wf[16];
 #pragma unroll
                 for (int a = 0; a < 4; ++a)
 #pragma unroll
-                    for (int q = 0; q < 4; ++q) w[a][q] += __shfl_xor_sync(0xffffffffu, w[a][q], o);
+                    for (int q = 0; q < 4; ++q) wf[a * 4 + q] = w[a][q];
+                warp_reduce_many<16>(wf, scr);
+#pragma unroll
+                for (int a = 0; a < 4; ++a)
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) w[a][q] = wf[a * 4 + q];
+            }
             T tt[16];
 #pragma unroll
             for (int k = 0; k < 16; ++k) tt[k] = Tb[b * 16 + k];
@@ -460,13 +515,13 @@ __device__ __forceinline__ void factor_panel_wb4(T* P, int RGP, int RG, int wp, 
             }
         }
     }
-    __syncthreads();  // every block applied: P's v columns are no longer read
+    gsync(G);  // every block applied: P's v columns are no longer read
 #pragma unroll
     for (int q = 0; q < 4; ++q)
         if (q < nc)
 #pragma unroll
             for (int i = 0; i < 8; ++i) P[(size_t)(cb + q) * RGP + padr<T>(lane + 32 * i)] = x[q][i];
-    __syncthreads();
+    gsync(G);
 }
 
 // ---------------------------------------------------------------------------
@@ -474,10 +529,10 @@ __device__ __forceinline__ void factor_panel_wb4(T* P, int RGP, int RG, int wp, 
 // 8 warps = 4-way split of the rows x 2 column halves; deterministic reduction.
 // ---------------------------------------------------------------------------
 template <typename T>
-__device__ __forceinline__ void gemm_vtc(const T* Vs, const T* Cs, int RGP, int R32, T* Wp, T* W) {
+__device__ __forceinline__ void gemm_vtc(const Grp& G, const T* Vs, const T* Cs, int RGP, int R32, T* Wp, T* W) {
     using V4 = typename Vec4<T>::type;
     constexpr int VN = Vec4<T>::n;
-    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int tid = G.tid, warp = tid >> 5, lane = tid & 31;
     const int ks = warp & 3, ch = warp >> 2;
     const int jg = lane & 7, cg = lane >> 3;
     const int chunk = R32 / 4;
@@ -506,7 +561,7 @@ __device__ __forceinline__ void gemm_vtc(const T* Vs, const T* Cs, int RGP, int 
     for (int a = 0; a < 4; ++a)
 #pragma unroll
         for (int b = 0; b < 4; ++b) Wp[(ks * 32 + jg + 8 * a) * kTS + 16 * ch + cg + 4 * b] = acc[a][b];
-    __syncthreads();
+    gsync(G);
     for (int e = tid; e < 32 * 32; e += kThreads) {
         const int jj = e >> 5, cc2 = e & 31;
         T sum = Wp[(0 * 32 + jj) * kTS + cc2];
@@ -515,7 +570,7 @@ __device__ __forceinline__ void gemm_vtc(const T* Vs, const T* Cs, int RGP, int 
         sum += Wp[(3 * 32 + jj) * kTS + cc2];
         W[jj * kTS + cc2] = sum;
     }
-    __syncthreads();
+    gsync(G);
 }
 
 // T (upper triangular, Tt[r*kTS+c] = T[r][c]) from G = V^T V (strict upper
@@ -523,9 +578,9 @@ __device__ __forceinline__ void gemm_vtc(const T* Vs, const T* Cs, int RGP, int 
 // T[0:j,j] = -tau_j T[0:j,0:j] G[0:j,j].  One warp; lane i keeps row i of T in
 // registers; 4 independent accumulation chains.
 template <typename T>
-__device__ __forceinline__ void build_t(const T* G, const T* tau_s, int wp, T* Tt) {
-    const int lane = threadIdx.x & 31;
-    if (threadIdx.x >= 32) return;
+__device__ __forceinline__ void build_t(const Grp& Gr, const T* G, const T* tau_s, int wp, T* Tt) {
+    const int lane = Gr.tid & 31;
+    if (Gr.tid >= 32) return;
     T row[32];
 #pragma unroll
     for (int j = 0; j < 32; ++j) {
@@ -547,13 +602,158 @@ __device__ __forceinline__ void build_t(const T* G, const T* tau_s, int wp, T* T
 }
 
 // C(RG x 32, in Cs) <- C - V (op(T) W) ; written straight to global rows.
+// ---------------------------------------------------------------------------
+// Tensor-core path of the trailing update (fp32): mma.sync m16n8k8 TF32 with
+// the 3xTF32 split (x = hi + lo, hi = tf32(x), lo = tf32(x - hi); a*b ~
+// ahi*bhi + ahi*blo + alo*bhi), fp32 accumulation.  Measured on this B200:
+// 276 TF/s TF32 dense -> ~92 TF/s 3xTF32, vs 71 TF/s FFMA; the point is the
+// ~5x lower shared-memory traffic per multiply-add (register fragments reused
+// across tiles), which frees the MIO pipe the panel factorization needs.
+// Used only for W = V^T C and C -= V W2 of the factorization's trailing
+// update: V, T (hence Q) stay exact fp32, so Q's orthogonality is unaffected;
+// the trailing matrix sees ~2^-22 relative product errors (backward error).
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void split_tf32(float x, uint32_t& hi, uint32_t& lo) {
+    uint32_t h, l;
+    asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(h) : "f"(x));
+    const float r = x - __uint_as_float(h);
+    asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(l) : "f"(r));
+    hi = h;
+    lo = l;
+}
+__device__ __forceinline__ void mma_tf32(float (&d)[4], const uint32_t (&a)[4], const uint32_t (&b)[2]) {
+    asm volatile(
+        "mma.sync.aligned.m16n8k8.row.col.f32.tf32.tf32.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+        "{%0,%1,%2,%3};"
+        : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
+        : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b[0]), "r"(b[1]));
+}
+__device__ __forceinline__ void mma_3xtf32(float (&d)[4], const uint32_t (&ah)[4], const uint32_t (&al)[4],
+                                           const uint32_t (&bh)[2], const uint32_t (&bl)[2]) {
+    mma_tf32(d, al, bh);
+    mma_tf32(d, ah, bl);
+    mma_tf32(d, ah, bh);
+}
+
+// W(32 x 32) = V^T C on tensor cores; same warp split and deterministic
+// 4-way reduction as gemm_vtc.
+__device__ __forceinline__ void gemm_vtc_mma(const Grp& G, const float* Vs, const float* Cs, int RGP, int R32,
+                                             float* Wp, float* W) {
+    const int warp = G.tid >> 5, lane = G.tid & 31;
+    const int ks = warp & 3, ch = warp >> 2;
+    const int g = lane >> 2, t = lane & 3;
+    const int chunk = R32 / 4;
+    const int rbeg = ks * chunk, rend = rbeg + chunk;
+    float acc[2][2][4];
+#pragma unroll
+    for (int a = 0; a < 2; ++a)
+#pragma unroll
+        for (int b = 0; b < 2; ++b)
+#pragma unroll
+            for (int e = 0; e < 4; ++e) acc[a][b][e] = 0.f;
+    for (int k0 = rbeg; k0 < rend; k0 += 8) {
+        const int p0 = padr<float>(k0 + t), p1 = padr<float>(k0 + t + 4);
+        uint32_t ah[2][4], al[2][4], bh[2][2], bl[2][2];
+#pragma unroll
+        for (int mt = 0; mt < 2; ++mt) {
+            const float* v0 = Vs + (size_t)(16 * mt + g) * RGP;
+            const float* v8 = v0 + 8 * (size_t)RGP;
+            split_tf32(v0[p0], ah[mt][0], al[mt][0]);
+            split_tf32(v8[p0], ah[mt][1], al[mt][1]);
+            split_tf32(v0[p1], ah[mt][2], al[mt][2]);
+            split_tf32(v8[p1], ah[mt][3], al[mt][3]);
+        }
+#pragma unroll
+        for (int nt = 0; nt < 2; ++nt) {
+            const float* c0 = Cs + (size_t)(16 * ch + 8 * nt + g) * RGP;
+            split_tf32(c0[p0], bh[nt][0], bl[nt][0]);
+            split_tf32(c0[p1], bh[nt][1], bl[nt][1]);
+        }
+#pragma unroll
+        for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+            for (int nt = 0; nt < 2; ++nt) mma_3xtf32(acc[mt][nt], ah[mt], al[mt], bh[nt], bl[nt]);
+    }
+#pragma unroll
+    for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+        for (int nt = 0; nt < 2; ++nt) {
+            const int jj = 16 * mt + g, c = 16 * ch + 8 * nt + 2 * t;
+            float* wr = Wp + (ks * 32 + jj) * kTS + c;
+            wr[0] = acc[mt][nt][0];
+            wr[1] = acc[mt][nt][1];
+            wr[8 * kTS] = acc[mt][nt][2];
+            wr[8 * kTS + 1] = acc[mt][nt][3];
+        }
+    gsync(G);
+    for (int e = G.tid; e < 32 * 32; e += kThreads) {
+        const int jj = e >> 5, c = e & 31;
+        float sum = Wp[(0 * 32 + jj) * kTS + c];
+        sum += Wp[(1 * 32 + jj) * kTS + c];
+        sum += Wp[(2 * 32 + jj) * kTS + c];
+        sum += Wp[(3 * 32 + jj) * kTS + c];
+        W[jj * kTS + c] = sum;
+    }
+    gsync(G);
+}
+
+// Cs(R32 x 32) <- Cs - V W2 on tensor cores (W2 in W, rows jj).  Warp w owns
+// row tiles {w, w + 8, ...} of 16 rows and all 4 column tiles.
+__device__ __forceinline__ void gemm2_mma(const Grp& G, const float* Vs, float* Cs, const float* W, int RGP,
+                                          int R32) {
+    const int warp = G.tid >> 5, lane = G.tid & 31;
+    const int g = lane >> 2, t = lane & 3;
+    // B fragments (-W2) for all 4 k-steps x 4 column tiles, split once
+    uint32_t bh[4][4][2], bl[4][4][2];
+#pragma unroll
+    for (int kk = 0; kk < 4; ++kk)
+#pragma unroll
+        for (int nt = 0; nt < 4; ++nt) {
+            split_tf32(-W[(8 * kk + t) * kTS + 8 * nt + g], bh[kk][nt][0], bl[kk][nt][0]);
+            split_tf32(-W[(8 * kk + t + 4) * kTS + 8 * nt + g], bh[kk][nt][1], bl[kk][nt][1]);
+        }
+    for (int mt = warp; mt < R32 / 16; mt += kWarps) {
+        const int m0 = 16 * mt;
+        const int r0 = padr<float>(m0 + g), r8 = padr<float>(m0 + g + 8);
+        float d[4][4];
+#pragma unroll
+        for (int nt = 0; nt < 4; ++nt) {
+            const float* c0 = Cs + (size_t)(8 * nt + 2 * t) * RGP;
+            d[nt][0] = c0[r0];
+            d[nt][1] = c0[RGP + r0];
+            d[nt][2] = c0[r8];
+            d[nt][3] = c0[RGP + r8];
+        }
+#pragma unroll
+        for (int kk = 0; kk < 4; ++kk) {
+            const float* va = Vs + (size_t)(8 * kk + t) * RGP;
+            const float* vb = va + 4 * (size_t)RGP;
+            uint32_t ah[4], al[4];
+            split_tf32(va[r0], ah[0], al[0]);
+            split_tf32(va[r8], ah[1], al[1]);
+            split_tf32(vb[r0], ah[2], al[2]);
+            split_tf32(vb[r8], ah[3], al[3]);
+#pragma unroll
+            for (int nt = 0; nt < 4; ++nt) mma_3xtf32(d[nt], ah, al, bh[kk][nt], bl[kk][nt]);
+        }
+#pragma unroll
+        for (int nt = 0; nt < 4; ++nt) {
+            float* c0 = Cs + (size_t)(8 * nt + 2 * t) * RGP;
+            c0[r0] = d[nt][0];
+            c0[RGP + r0] = d[nt][1];
+            c0[r8] = d[nt][2];
+            c0[RGP + r8] = d[nt][3];
+        }
+    }
+}
+
 template <typename T>
-__device__ __forceinline__ void apply_block(const T* Vs, const T* Cs, const T* Tt, T* W, int RGP, int R32,
+__device__ __forceinline__ void apply_block(const Grp& G, const T* Vs, const T* Cs, const T* Tt, T* W, int RGP, int R32,
                                             int RG, int wp, int trans, const NodeRows& nr, T* C,
                                             int64_t ldc, int64_t cb0, int ncb) {
     using V4 = typename Vec4<T>::type;
     constexpr int VN = Vec4<T>::n;
-    const int tid = threadIdx.x;
+    const int tid = G.tid;
     // W2 = op(T) W: thread (column c, rows jj = jg + 8q); T is zero below its
     // diagonal, so full unrolled sums need no bounds.
     T w2[4];
@@ -584,10 +784,13 @@ __device__ __forceinline__ void apply_block(const T* Vs, const T* Cs, const T* T
             }
         }
     }
-    __syncthreads();
+    gsync(G);
 #pragma unroll
     for (int q = 0; q < 4; ++q) W[((tid >> 5) + 8 * q) * kTS + (tid & 31)] = w2[q];
-    __syncthreads();
+    gsync(G);
+    if constexpr (sizeof(T) == 4) {
+        gemm2_mma(G, Vs, const_cast<T*>(Cs), W, RGP, R32);
+    } else {
     const int nq = R32 / 4;
     for (int u = tid; u < nq * 4; u += kThreads) {
         const int q = u % nq, cgrp = u / nq;
@@ -637,7 +840,8 @@ __device__ __forceinline__ void apply_block(const T* Vs, const T* Cs, const T* T
             }
         }
     }
-    __syncthreads();
+    }
+    gsync(G);
     {
         const int warp = tid >> 5, lane = tid & 31;
         for (int c = warp; c < ncb; c += kWarps) {
@@ -646,16 +850,16 @@ __device__ __forceinline__ void apply_block(const T* Vs, const T* Cs, const T* T
             for (int r = lane; r < RG; r += 32) ccol[gathered_row(nr, r)] = cs[padr<T>(r)];
         }
     }
-    __syncthreads();
+    gsync(G);
 }
 
 template <typename T>
-__device__ __forceinline__ void stage_cols(T* S, int RGP, int R32, const T* M, int64_t ld, int64_t col0,
+__device__ __forceinline__ void stage_cols(const Grp& G, T* S, int RGP, int R32, const T* M, int64_t ld, int64_t col0,
                                            int ncol, const NodeRows& nr, int RG, bool mask_panel, int p) {
     // Every thread issues all of its loads before the first store (memory-level
     // parallelism: up to 32 L2/HBM requests in flight per thread), in halves
     // of 16 for fp64 to bound register use.
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int warp = G.tid >> 5, lane = G.tid & 31;
     constexpr int NA = sizeof(T) == 4 ? 4 : 2;  // columns per batch per warp
 #pragma unroll
     for (int a0 = 0; a0 < 4; a0 += NA) {
@@ -701,6 +905,7 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
     T* W = Tt + 32 * kTS;
     T* tau_s = W + 32 * kTS;
     __shared__ int s_task;
+    const Grp G0{(int)threadIdx.x, 0};
     int* ticket = sync;
     int* flags = sync + 32;  // [L][npan]
     const int64_t leaf_tasks = do_leaves ? g.P : 0;  // one task per chain of K tiles
@@ -771,11 +976,11 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
             const int R32 = (RG + 31) & ~31;
             const int64_t c0 = g.col0 + 32 * p;
             // ---- panel: stage, factor, store R/V, T ------------------------
-            stage_cols(P, RGP, R32, A, g.lda, c0, wp, nr, RG, true, p);
+            stage_cols(G0, P, RGP, R32, A, g.lda, c0, wp, nr, RG, true, p);
             if (threadIdx.x < 32) tau_s[threadIdx.x] = T(0);
             __syncthreads();
             CAQR_PROF(2);
-            factor_panel_wb4<T>(P, RGP, RG, wp, tau_s, Wp);
+            factor_panel_wb4<T>(G0, P, RGP, RG, wp, tau_s, Wp, Cs);
             CAQR_PROF(3);
             {
                 const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -798,8 +1003,8 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
             }
             __syncthreads();
             CAQR_PROF(4);
-            gemm_vtc(P, P, RGP, R32, Wp, W);  // G = V^T V
-            build_t(W, tau_s, wp, Tt);
+            gemm_vtc(G0, P, P, RGP, R32, Wp, W);  // G = V^T V
+            build_t(G0, W, tau_s, wp, Tt);
             __syncthreads();
             {
                 T* tb = Tws + nr.tblk * (kPW * kPW);
@@ -813,12 +1018,15 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
             const int64_t tfirst = c0 + 32, tend = g.col0 + g.ncols;
             for (int64_t cb0 = tfirst; cb0 < tend; cb0 += 32) {
                 const int ncb = (int)(tend - cb0 < 32 ? tend - cb0 : 32);
-                stage_cols(Cs, RGP, R32, static_cast<const T*>(A), g.lda, cb0, ncb, nr, RG, false, p);
+                stage_cols(G0, Cs, RGP, R32, static_cast<const T*>(A), g.lda, cb0, ncb, nr, RG, false, p);
                 __syncthreads();
                 CAQR_PROF(6);
-                gemm_vtc(P, Cs, RGP, R32, Wp, W);
+                if constexpr (sizeof(T) == 4)
+                    gemm_vtc_mma(G0, P, Cs, RGP, R32, Wp, W);
+                else
+                    gemm_vtc(G0, P, Cs, RGP, R32, Wp, W);
                 CAQR_PROF(7);
-                apply_block(P, Cs, Tt, W, RGP, R32, RG, wp, 1, nr, A, g.lda, cb0, ncb);
+                apply_block(G0, P, Cs, Tt, W, RGP, R32, RG, wp, 1, nr, A, g.lda, cb0, ncb);
                 CAQR_PROF(8);
             }
             // ---- publish ----------------------------------------------------------
@@ -832,6 +1040,197 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
     if (prof && threadIdx.x == 0)
         for (int k = 0; k < 12; ++k) atomicAdd(prof + k, pacc[k]);
 #undef CAQR_PROF
+}
+
+}  // namespace caqr
+
+// ===========================================================================
+// Look-ahead variant (fp32): one CTA of 512 threads per SM, two roles.
+//   F (warps 0-7, named barrier 1): stage + factor the NEXT panel (WB4), its
+//     T, and write it out;
+//   U (warps 8-15, named barrier 2): apply the CURRENT panel's block
+//     reflector to the node's trailing column blocks.
+// Per panel p: U first updates block p+1 (the next panel's columns; F waits),
+// then F factors panel p+1 while U updates blocks >= p+2 -- the classic
+// look-ahead, so the latency-bound panel factorization overlaps the GEMM-like
+// trailing update instead of alternating with it.
+// ===========================================================================
+namespace caqr {
+
+template <typename T>
+struct LaSmem {
+    T *PA, *PB, *Cs, *Wp, *WpF, *TA, *TB, *WU, *WF, *tauA, *tauB, *TbF, *scrF;
+};
+
+template <typename T>
+__host__ __device__ inline size_t la_smem_elems(int RGP) {
+    return 3 * 32 * (size_t)RGP + 2 * 4 * 32 * kTS + 4 * 32 * kTS + 64 + 128 + kWarps * (32 * 20 + 16);
+}
+template <typename T>
+inline size_t la_smem_bytes() {
+    return sizeof(T) * la_smem_elems<T>(fused_col_stride<T>(kFusedMaxRows)) + 64;
+}
+
+template <typename T>
+__device__ __forceinline__ void la_factor_panel(const Grp& GF, const Geom& g, T* A, T* Tws, int level,
+                                                int64_t node, int kt, int p, T* P, T* Tt, T* tau, T* WpF,
+                                                T* WF, T* Tb, T* scr, int RGP) {
+    const int wp = min(kPW, g.ncols - 32 * p);
+    const NodeRows nr = node_rows(g, level, node, p, wp, kt);
+    const int RG = nr.n0 + nr.n1;
+    const int R32 = (RG + 31) & ~31;
+    const int64_t c0 = g.col0 + 32 * p;
+    stage_cols(GF, P, RGP, R32, static_cast<const T*>(A), g.lda, c0, wp, nr, RG, true, p);
+    if (GF.tid < 32) tau[GF.tid] = T(0);
+    gsync(GF);
+    factor_panel_wb4<T>(GF, P, RGP, RG, wp, tau, Tb, scr);
+    {
+        const int warp = GF.tid >> 5, lane = GF.tid & 31;
+        for (int jj = warp; jj < 32; jj += kWarps) {
+            T* col = A + (c0 + jj) * g.lda;
+            T* pc = P + (size_t)jj * RGP;
+            for (int r = lane; r < R32; r += 32) {
+                const bool in = r < RG && jj < wp;
+                const T val = pc[padr<T>(r)];
+                if (in && panel_entry_stored(nr, r, jj, p)) col[gathered_row(nr, r)] = val;
+                pc[padr<T>(r)] = in ? v_entry<T>(nr, r, jj, p, val) : T(0);
+            }
+        }
+    }
+    gsync(GF);
+    gemm_vtc(GF, P, P, RGP, R32, WpF, WF);  // G = V^T V
+    build_t(GF, WF, tau, wp, Tt);
+    gsync(GF);
+    T* tb = Tws + nr.tblk * (kPW * kPW);
+    for (int e = GF.tid; e < kPW * kPW; e += kThreads) tb[e] = Tt[(e & 31) * kTS + (e >> 5)];
+}
+
+template <typename T>
+__device__ __forceinline__ void la_update_block(const Grp& GU, const Geom& g, T* A, const NodeRows& nr, int p,
+                                                int wp, int64_t cb0, int ncb, const T* P, const T* Tt, T* Cs,
+                                                T* Wp, T* WU, int RGP) {
+    const int RG = nr.n0 + nr.n1;
+    const int R32 = (RG + 31) & ~31;
+    stage_cols(GU, Cs, RGP, R32, static_cast<const T*>(A), g.lda, cb0, ncb, nr, RG, false, p);
+    gsync(GU);
+    if constexpr (sizeof(T) == 4)
+        gemm_vtc_mma(GU, P, Cs, RGP, R32, Wp, WU);
+    else
+        gemm_vtc(GU, P, Cs, RGP, R32, Wp, WU);
+    apply_block(GU, P, Cs, Tt, WU, RGP, R32, RG, wp, 1, nr, A, g.lda, cb0, ncb);
+}
+
+template <typename T>
+__global__ void __launch_bounds__(2 * kThreads, 1)
+tsqr_la_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int nlevels, int do_leaves) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int RGP = fused_col_stride<T>(kFusedMaxRows);
+    T* base = reinterpret_cast<T*>(smem_raw);
+    T* PA = base;
+    T* PB = PA + 32 * (size_t)RGP;
+    T* Cs = PB + 32 * (size_t)RGP;
+    T* Wp = Cs + 32 * (size_t)RGP;
+    T* WpF = Wp + 4 * 32 * kTS;
+    T* TA = WpF + 4 * 32 * kTS;
+    T* TB = TA + 32 * kTS;
+    T* WU = TB + 32 * kTS;
+    T* WF = WU + 32 * kTS;
+    T* tauA = WF + 32 * kTS;
+    T* tauB = tauA + 32;
+    T* TbF = tauB + 32;
+    T* scrF = TbF + 128;
+    __shared__ int s_task;
+    const bool isF = threadIdx.x < kThreads;
+    const Grp GF{(int)threadIdx.x, 1}, GU{(int)threadIdx.x - kThreads, 2};
+    int* ticket = sync;
+    int* flags = sync + 32;
+    const int64_t leaf_tasks = do_leaves ? g.P : 0;
+    int64_t total = leaf_tasks;
+    for (int l = 0; l < nlevels; ++l) {
+        const int64_t h = int64_t(1) << l;
+        total += (g.P - 1 >= h) ? (g.P - 1 - h) / (2 * h) + 1 : 0;
+    }
+    for (;;) {
+        __syncthreads();
+        if (threadIdx.x == 0) s_task = atomicAdd(ticket, 1);
+        __syncthreads();
+        const int64_t task = s_task;
+        if (task >= total) break;
+        int level = -1;
+        int64_t node = task;
+        if (task >= leaf_tasks) {
+            node = task - leaf_tasks;
+            level = 0;
+            for (;;) {
+                const int64_t h = int64_t(1) << level;
+                const int64_t nm = (g.P - 1 >= h) ? (g.P - 1 - h) / (2 * h) + 1 : 0;
+                if (node < nm) break;
+                node -= nm;
+                ++level;
+            }
+        }
+        int64_t slot_a, slot_b = -1;
+        int ver_a = 0, ver_b = 0;
+        if (level < 0) {
+            slot_a = node;
+        } else {
+            slot_a = node << (level + 1);
+            slot_b = slot_a + (int64_t(1) << level);
+            ver_a = expected_version(slot_a, level, g.P, do_leaves);
+            ver_b = expected_version(slot_b, level, g.P, do_leaves);
+        }
+        const int my_ver = level < 0 ? 1 : level + 2;
+        const int64_t ntile = level < 0 ? min(g.K, g.L - node * g.K) : 1;
+        auto wait_children = [&](int p) {  // F thread 0; then F barrier
+            if (level >= 0 && GF.tid == 0) {
+                const int* fa = flags + slot_a * g.npan + p;
+                const int* fb = flags + slot_b * g.npan + p;
+                while (ld_acquire(fa) < ver_a) __nanosleep(64);
+                while (ld_acquire(fb) < ver_b) __nanosleep(64);
+            }
+            gsync(GF);
+        };
+        for (int kt = 0; kt < ntile; ++kt) {
+            T *Pc = PA, *Pn = PB, *Tc = TA, *Tn = TB, *tc = tauA, *tn = tauB;
+            if (isF) {
+                wait_children(0);
+                la_factor_panel(GF, g, A, Tws, level, node, kt, 0, Pc, Tc, tc, WpF, WF, TbF, scrF, RGP);
+            }
+            __syncthreads();
+            for (int p = 0; p < g.npan; ++p) {
+                const int wp = min(kPW, g.ncols - 32 * p);
+                const bool has_next = p + 1 < g.npan;
+                const NodeRows nr = node_rows(g, level, node, p, wp, kt);
+                const int64_t c0 = g.col0 + 32 * p, tend = g.col0 + g.ncols;
+                // step 1: U brings the next panel's columns up to date
+                if (!isF && has_next) {
+                    const int64_t cb0 = c0 + 32;
+                    la_update_block(GU, g, A, nr, p, wp, cb0, (int)(tend - cb0 < 32 ? tend - cb0 : 32), Pc, Tc, Cs,
+                                    Wp, WU, RGP);
+                }
+                __syncthreads();
+                // step 2: F factors panel p+1 while U updates the far blocks
+                if (isF) {
+                    if (has_next) {
+                        wait_children(p + 1);
+                        la_factor_panel(GF, g, A, Tws, level, node, kt, p + 1, Pn, Tn, tn, WpF, WF, TbF, scrF,
+                                        RGP);
+                    }
+                } else {
+                    for (int64_t cb0 = c0 + 64; cb0 < tend; cb0 += 32)
+                        la_update_block(GU, g, A, nr, p, wp, cb0, (int)(tend - cb0 < 32 ? tend - cb0 : 32), Pc, Tc,
+                                        Cs, Wp, WU, RGP);
+                }
+                __threadfence();
+                __syncthreads();
+                if (threadIdx.x == 0 && kt == ntile - 1) st_release(flags + slot_a * g.npan + p, my_ver);
+                T* t;
+                t = Pc; Pc = Pn; Pn = t;
+                t = Tc; Tc = Tn; Tn = t;
+                t = tc; tc = tn; tn = t;
+            }
+        }
+    }
 }
 
 }  // namespace caqr

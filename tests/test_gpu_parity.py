@@ -312,3 +312,10 @@ def test_fused_and_split_agree(caqr, monkeypatch):
     monkeypatch.setenv("CAQR_FUSED", "0")
     R2, _, _, _ = gpu_qr(caqr, A, opts, want_q=False)
     assert np.linalg.norm(R1 - R2) / np.linalg.norm(R1) <= 1e-5
+
+
+def test_lookahead_kernel(caqr, monkeypatch):
+    """The look-ahead (two-role) fp32 fused kernel: same plan, same R to rounding."""
+    monkeypatch.setenv("CAQR_LA", "1")
+    A = workloads.gaussian(70000, 192, seed=12)
+    check_against_oracle(caqr, A, opts=caqr.make_opts(leaf_rows=224), C_cols=2)
