@@ -15,6 +15,7 @@
 #include "../../include/caqr.h"
 #include "tsqr_fused.cuh"
 #include "tsqr_kernels.cuh"
+#include "tsqr_skinny.cuh"
 
 namespace caqr {
 
@@ -23,9 +24,9 @@ static thread_local int g_last_cuda_error = 0;
 // ---- launch tracing (diagnostics: per-launch CUDA events on the launching
 // stream + host-computed algorithmic flops/bytes; see caqr_trace_begin) -------
 enum KernelId { K_PANEL_FACTOR = 0, K_PANEL_UPDATE = 1, K_EXTRACT_R = 2, K_SET_IDENTITY = 3,
-                K_TSQR_FUSED = 4, K_NUM = 5 };
+                K_TSQR_FUSED = 4, K_TSQR_SKINNY = 5, K_NUM = 6 };
 static const char* const kKernelNames[K_NUM] = {"panel_factor", "panel_update", "extract_r",
-                                                "set_identity", "tsqr_fused"};
+                                                "set_identity", "tsqr_fused", "tsqr_skinny"};
 struct Trace {
     std::mutex mu;
     bool on = false;
@@ -65,6 +66,8 @@ struct Plan {
     int64_t b = 0;   // leaf height
     int64_t nb = 0;  // panel-group width
     int64_t ngroups = 0;
+    int64_t chain_target = 296;  // chains per group (tree leaves)
+    bool skinny = false;         // warp-per-task skinny kernel (fp32, n <= 16)
 };
 
 static inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
@@ -78,7 +81,15 @@ static int make_plan(int64_t m, int64_t n, int dtype, const caqr_opts* o, int op
     int64_t nb = (o && o->panel_cols > 0) ? o->panel_cols : (n <= kMaxGroup ? n : 64);
     if (nb > kMaxGroup) return -opt_pos;
     nb = std::max<int64_t>(1, std::min(nb, std::max<int64_t>(n, 1)));
-    int64_t b = (o && o->leaf_rows > 0) ? o->leaf_rows : (nb <= kFusedLeaf ? kFusedLeaf : kMaxLeaf);
+    // skinny fp32 panels (n <= 16, one group): one warp per task, 256-row (n <= 8)
+    // or 128-row (n <= 16) tiles, ~2,000 chains (see tsqr_skinny.cuh)
+    // (only for genuinely tall inputs: below ~256k rows the block kernel's
+    // fewer, larger tasks win, e.g. 4096 x 16: 0.13 ms vs 0.26 ms measured)
+    pl->skinny = dtype == CAQR_F32 && n <= 16 && nb >= n && m >= (int64_t(1) << 18);
+    pl->chain_target = pl->skinny ? 2048 : kChainTarget;
+    int64_t b = (o && o->leaf_rows > 0) ? o->leaf_rows
+                                        : (pl->skinny ? (n <= 8 ? 256 : 128)
+                                                      : (nb <= kFusedLeaf ? kFusedLeaf : kMaxLeaf));
     if (b % 32 != 0 || b > kMaxLeaf) return -opt_pos;
     b = std::max(b, round_up(nb, 32));
     if (b > kMaxLeaf) return -opt_pos;
@@ -98,7 +109,7 @@ static Geom group_geom(const Plan& pl, int64_t g, int64_t lda) {
     G.npan = (int32_t)ceil_div(G.ncols, kPW);
     G.b = pl.b;
     G.L = std::max<int64_t>(1, ceil_div(G.mrows, pl.b));
-    G.K = ceil_div(G.L, kChainTarget);
+    G.K = ceil_div(G.L, pl.chain_target);
     G.P = ceil_div(G.L, G.K);
     G.bm = G.K * G.b;
     return G;
@@ -346,6 +357,11 @@ static int launch_fused(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, 
 
 // CAQR_FUSED=0 forces the split (one launch per level and panel) path; read
 // on every call so tests can compare both paths in one process.
+static inline int skinny_policy() {
+    const char* e = getenv("CAQR_SKINNY");
+    return (e && e[0] == '0') ? 0 : 1;
+}
+
 static inline int fused_policy() {
     const char* e = getenv("CAQR_FUSED");
     return (e && e[0] == '0') ? 0 : 1;
@@ -353,8 +369,54 @@ static inline int fused_policy() {
 
 // TSQR of one panel group (Fig. 4 minus the trailing update): every leaf's
 // panels (factor + intra-group trailing update), then every tree level.
+// Skinny groups (fp32, n <= 16): the warp-per-task kernel; true if launched.
+template <typename T>
+static int launch_skinny(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, cudaStream_t s, bool* done) {
+    *done = false;
+    if constexpr (sizeof(T) == 4) {
+        const int nr_need = (int)ceil_div(G.ncols + G.b, 32);
+        const bool fit8 = G.ncols <= 8 && nr_need <= 9, fit16 = G.ncols <= 16 && nr_need <= 5;
+        if (!fit8 && !fit16) return 0;
+        const int nl = tree_levels(G.P);
+        int64_t total = do_leaves ? G.P : 0;
+        for (int lv = 0; lv < nl; ++lv) total += merges_at(G.P, lv);
+        if (total <= 0) {
+            *done = true;
+            return 0;
+        }
+        cudaError_t e = cudaMemsetAsync(sync, 0, group_sync_bytes(G), s);
+        if (e == cudaSuccess) {
+            const int64_t warps = std::min<int64_t>(total, (int64_t)num_sms() * 16);
+            const unsigned grid = (unsigned)ceil_div(warps, kSkinnyWarps);
+            double fl = 0, by = 0;
+            if (g_trace.on) {
+                const double mr = (double)G.mrows, nc = (double)G.ncols;
+                fl = 2.0 * mr * nc * nc - 2.0 / 3.0 * nc * nc * nc;
+                by = 2.0 * mr * nc * sizeof(T);
+            }
+            TraceScope ts(K_TSQR_SKINNY, fl, by, s);
+            if (fit8)
+                tsqr_skinny_kernel<8, 9><<<grid, 32 * kSkinnyWarps, 0, s>>>(G, A, Tws, sync, nl, do_leaves ? 1 : 0);
+            else
+                tsqr_skinny_kernel<16, 5><<<grid, 32 * kSkinnyWarps, 0, s>>>(G, A, Tws, sync, nl, do_leaves ? 1 : 0);
+            e = cudaGetLastError();
+        }
+        if (e != cudaSuccess) {
+            g_last_cuda_error = (int)e;
+            return CAQR_ERR_CUDA;
+        }
+        *done = true;
+    }
+    return 0;
+}
+
 template <typename T>
 static int factor_group(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, cudaStream_t s) {
+    if (fused_policy() && G.npan == 1 && G.ncols <= 16 && skinny_policy()) {
+        bool done = false;
+        const int rc = launch_skinny<T>(G, A, Tws, sync, do_leaves, s, &done);
+        if (rc || done) return rc;
+    }
     if (fused_policy() && fused_ok(G)) return launch_fused<T>(G, A, Tws, sync, do_leaves, s);
     int rc = 0;
     if (do_leaves) {
@@ -733,7 +795,7 @@ int caqr_plan_info(int64_t m, int64_t n, int dtype, const caqr_opts* opts, int64
     for (int64_t g = 0; g < pl.ngroups; ++g) {
         const Geom Gg = group_geom(pl, g, m);
         const int nl = tree_levels(Gg.P);
-        if (fused_ok(Gg))
+        if (fused_ok(Gg) || (pl.skinny && Gg.npan == 1))
             launches += 1;
         else
             launches += (int64_t)(nl + Gg.K) * (2 * Gg.npan - 1);

@@ -349,7 +349,10 @@ panel_update_kernel(Geom g, const T* A, const T* __restrict__ Tws, int level, in
     }
     {
         const T* tb = Tws + nr.tblk * (kPW * kPW);
-        for (int e = tid; e < kPW * kPW; e += kThreads) Tt[(e & 31) * kTS + (e >> 5)] = tb[e];
+        // only the wp x wp part of a T block is meaningful (the skinny kernel
+        // writes nothing else)
+        for (int e = tid; e < kPW * kPW; e += kThreads)
+            Tt[(e & 31) * kTS + (e >> 5)] = ((e & 31) < wp && (e >> 5) < wp) ? tb[e] : T(0);
     }
     __syncthreads();
 

@@ -39,7 +39,8 @@ def test_workspace_bytes(L):
     # plus the fused kernel's ticket + (slot, panel) flags: (32 + L*npan) ints, 256-B rounded
     def ws(L, npan, es):
         return 2 * L * npan * 1024 * es + -(-(32 + L * npan) * 4 // 256) * 256
-    # default tile height 224 (n <= 224): 4096 rows -> 19 tiles; 1M rows -> 4465 tiles
+    # default tile height 224 (n <= 224): 4096 rows -> 19 tiles, 1M rows -> 4465 tiles;
+    # skinny fp32 (n <= 16, m >= 2^18: warp-per-task kernel) uses 256/128-row tiles
     assert caqr.caqr_workspace_bytes(4096, 16) == ws(19, 1, 4)
     assert caqr.caqr_workspace_bytes(4096, 16, caqr.CAQR_F64) == ws(19, 1, 8)
     assert caqr.caqr_workspace_bytes(1_000_000, 192) == ws(4465, 6, 4)
@@ -60,6 +61,8 @@ def test_plan_info(L):
     assert p["panel_cols"] == 64 and p["groups"] == 128
     p = caqr.caqr_plan_info(4096, 16, 0, caqr.make_opts(leaf_rows=128))
     assert p["leaf_rows"] == 128 and p["leaves"] == 32 and p["tree_levels"] == 5
+    p = caqr.caqr_plan_info(4_000_000, 8)  # skinny: 256-row tiles, ~2048 chains
+    assert p["leaf_rows"] == 256 and p["leaves"] == 15625 and p["chains"] == 1954 and p["launches"] == 2
 
 
 def test_info_codes_without_gpu(L):

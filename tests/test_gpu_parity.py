@@ -319,3 +319,22 @@ def test_lookahead_kernel(caqr, monkeypatch):
     monkeypatch.setenv("CAQR_LA", "1")
     A = workloads.gaussian(70000, 192, seed=12)
     check_against_oracle(caqr, A, opts=caqr.make_opts(leaf_rows=224), C_cols=2)
+
+
+@pytest.mark.parametrize("m,n", [(600_000, 16), (2_100_000, 8), (530_000, 3)])
+def test_skinny_chains(caqr, m, n):
+    """Skinny fp32 panels (n <= 16) go to the warp-per-task kernel; with more
+    tiles than its 2048-chain target the tiles form chains."""
+    info = caqr.caqr_plan_info(m, n)
+    assert info["chains"] < info["leaves"]
+    A = workloads.gaussian(m, n, seed=n)
+    check_against_oracle(caqr, A, C_cols=2)
+
+
+def test_skinny_vs_block_kernel(caqr, monkeypatch):
+    """Warp-per-task and block kernels on the same plan agree to rounding."""
+    A = workloads.gaussian(300_000, 12, seed=3)
+    R1, _, _, _ = gpu_qr(caqr, A, want_q=False)
+    monkeypatch.setenv("CAQR_SKINNY", "0")
+    R2, _, _, _ = gpu_qr(caqr, A, want_q=False)
+    assert np.linalg.norm(R1 - R2) / np.linalg.norm(R1) <= 1e-5
