@@ -32,7 +32,9 @@
  *   - Return value: LAPACK "info".  0 = success; -i = argument i is illegal (the
  *     call does nothing); CAQR_ERR_CUDA (1) = a CUDA launch failed (see
  *     caqr_last_cuda_error); CAQR_ERR_NCCL (2) = an NCCL call failed.
- *     m = 0 or n = 0 is a quick return with 0.  NaN/Inf are not checked; they
+ *     m = 0 or n = 0 is a quick return with 0 (dimensions and leading
+ *     dimensions are checked first, pointers only when there is work, as
+ *     LAPACK never dereferences them then).  NaN/Inf are not checked; they
  *     propagate as in LAPACK.
  *   - Householder convention (reading S1): LAPACK xLARFG
  *     (beta = -sign(alpha)||x||, v(head) = 1, tau = (beta-alpha)/beta).  R_jj may be

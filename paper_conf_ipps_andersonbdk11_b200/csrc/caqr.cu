@@ -489,16 +489,17 @@ static int launch_extract_r(int64_t n, const T* A, int64_t lda, T* R, int64_t ld
 template <typename T>
 static int factor_impl(int64_t m, int64_t n, T* A, int64_t lda, T* R, int64_t ldr, void* ws,
                        size_t ws_bytes, const caqr_opts* opts, cudaStream_t s, int dtype) {
+    // dimensions first; LAPACK-style quick return before any pointer is used
     if (m < 0) return -1;
     if (n < 0 || n > m) return -2;
-    if (!A) return -3;
     if (lda < std::max<int64_t>(1, m)) return -4;
-    if (!R) return -5;
     if (ldr < std::max<int64_t>(1, n)) return -6;
     Plan pl;
     int rc = make_plan(m, n, dtype, opts, 9, &pl);
     if (rc) return rc;
     if (m == 0 || n == 0) return 0;
+    if (!A) return -3;
+    if (!R) return -5;
     if (!ws) return -7;
     if (ws_bytes < plan_ws_bytes(pl)) return -8;
     char* wsb = static_cast<char*>(ws);
@@ -522,15 +523,15 @@ static int apply_impl(int64_t m, int64_t n, const T* A, int64_t lda, const void*
                       int trans) {
     if (m < 0) return -1;
     if (n < 0 || n > m) return -2;
-    if (!A) return -3;
     if (lda < std::max<int64_t>(1, m)) return -4;
     if (k < 0) return -6;
-    if (!C) return -7;
     if (ldc < std::max<int64_t>(1, m)) return -8;
     Plan pl;
     int rc = make_plan(m, n, dtype, opts, 9, &pl);
     if (rc) return rc;
     if (m == 0 || n == 0 || k == 0) return 0;
+    if (!A) return -3;
+    if (!C) return -7;
     if (!ws) return -5;
     const T* base = static_cast<const T*>(ws);
     // group offsets into the workspace
@@ -559,11 +560,11 @@ static int form_q_impl(int64_t m, int64_t n, const T* A, int64_t lda, const void
                        int64_t ldq, const caqr_opts* opts, cudaStream_t s, int dtype) {
     if (m < 0) return -1;
     if (n < 0 || n > m) return -2;
-    if (!A) return -3;
     if (lda < std::max<int64_t>(1, m)) return -4;
-    if (!Q) return -6;
     if (ldq < std::max<int64_t>(1, m)) return -7;
     if (m == 0 || n == 0) return 0;
+    if (!A) return -3;
+    if (!Q) return -6;
     if (!ws) return -5;
     dim3 grid((unsigned)std::min<int64_t>(ceil_div(m, 256), 1024), (unsigned)n);
     cudaError_t e;

@@ -338,3 +338,70 @@ def test_skinny_vs_block_kernel(caqr, monkeypatch):
     monkeypatch.setenv("CAQR_SKINNY", "0")
     R2, _, _, _ = gpu_qr(caqr, A, want_q=False)
     assert np.linalg.norm(R1 - R2) / np.linalg.norm(R1) <= 1e-5
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64], ids=["f32", "f64"])
+def test_leading_dimensions(caqr, dtype):
+    """lda > m (A is a row-slice view of a taller buffer) and ldc > m for Q^T C."""
+    m, n, pad = 5000, 40, 77
+    tdt = torch.float32 if dtype == np.float32 else torch.float64
+    A = workloads.gaussian(m, n, seed=21, dtype=dtype)
+    big = caqr.colmajor_empty(m + pad, n, tdt)
+    big.zero_()
+    Av = big[:m]  # column-major view, stride (1, m + pad)
+    assert Av.stride(1) == m + pad
+    Av.copy_(torch.from_numpy(A))
+    R, ws = caqr.caqr_factor(Av)
+    Q = caqr.caqr_form_q(Av, ws)
+    Cbig = caqr.colmajor_empty(m + 13, 3, tdt)
+    C0 = workloads.gaussian(m, 3, seed=22, dtype=dtype)
+    Cv = Cbig[:m]
+    Cv.copy_(torch.from_numpy(C0))
+    caqr.caqr_apply_qt(Av, ws, Cv)
+    torch.cuda.synchronize()
+    bd = BOUNDS[dtype]
+    R64, Q64 = R.cpu().double().numpy(), Q.cpu().double().numpy()
+    assert np.linalg.norm(A - Q64 @ R64) / np.linalg.norm(A) <= bd["res"]
+    np.testing.assert_allclose(Cv.cpu().double().numpy()[:n], Q64.T @ C0, atol=50 * bd["res"] * np.abs(C0).max())
+    # rows below m of the padded buffer are untouched
+    assert torch.count_nonzero(big[m:]).item() == 0
+
+
+def test_empty_and_degenerate_shapes(caqr):
+    """m = n = 0 and n = 0 are quick returns; a zero matrix gives R = 0, tau = 0."""
+    A = caqr.colmajor_empty(10, 0)
+    R, ws = caqr.caqr_factor(A)
+    assert R.shape == (0, 0)
+    A = caqr.colmajor_empty(0, 0)
+    R, ws = caqr.caqr_factor(A)
+    Z = np.zeros((3000, 24), np.float32)
+    R, Q, _, _ = gpu_qr(caqr, Z)
+    assert np.all(R == 0)
+    # Q of a zero matrix is [I; 0] (every reflector is the identity)
+    assert np.array_equal(Q, np.eye(3000, 24))
+
+
+def test_chains_fp64(caqr):
+    A = workloads.gaussian(70000, 96, seed=31, dtype=np.float64)
+    opts = caqr.make_opts(leaf_rows=128)
+    assert caqr.caqr_plan_info(70000, 96, 1, opts)["chains"] < 547
+    check_against_oracle(caqr, A, opts=opts, C_cols=2)
+
+
+def test_max_single_gpu_size_properties(caqr):
+    """Config C4' (8,000,000 x 192 fp32, 6.1 GB) factored on one GPU: column
+    norms of R equal those of A and R^T R = A^T A (computed in fp64)."""
+    m, n = 8_000_000, 192
+    A = workloads.device_gaussian(m, n, seed=5, dtype=torch.float32, device="cuda").t()
+    G = torch.zeros((n, n), dtype=torch.float64, device="cuda")
+    cn = torch.zeros(n, dtype=torch.float64, device="cuda")
+    for s0 in range(0, m, 1_000_000):
+        blk = A[s0:s0 + 1_000_000].double()
+        G += blk.t() @ blk
+        cn += (blk * blk).sum(0)
+        del blk
+    R, ws = caqr.caqr_factor(A)
+    torch.cuda.synchronize()
+    R64 = R.double()
+    assert (torch.abs(torch.linalg.norm(R64, dim=0) - cn.sqrt()) / cn.sqrt()).max().item() <= 1e-4
+    assert (torch.linalg.norm(R64.t() @ R64 - G) / torch.linalg.norm(G)).item() <= 2e-4
