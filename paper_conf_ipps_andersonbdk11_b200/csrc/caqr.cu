@@ -259,20 +259,35 @@ static int launch_factor(const Geom& G, T* A, T* Tws, int level, int p, int kt, 
 template <typename T>
 static int launch_update(const Geom& G, const T* A, const T* Tws, int level, int p, int kt,
                          int64_t nodes, T* C, int64_t ldc, int64_t cfirst, int64_t ccount, int trans,
-                         cudaStream_t s) {
+                         cudaStream_t s, bool mma = false) {
     if (nodes <= 0 || ccount <= 0) return 0;
     const int wp = std::min<int>(kPW, G.ncols - 32 * p);
     const int rgmax = level < 0 ? (kt == 0 ? (int)std::min<int64_t>(G.b, G.mrows) : wp + (int)G.b)
                                 : 2 * wp + 32 * p;
     const size_t smem = panel_update_smem<T>(rgmax);
-    cudaError_t e = allow_smem(panel_update_kernel<T>, smem);
+    const bool use_mma = mma && sizeof(T) == 4;
+    cudaError_t e = cudaSuccess;
+    if constexpr (sizeof(T) == 4)
+        e = use_mma ? allow_smem(panel_update_kernel<T, true>, smem) : allow_smem(panel_update_kernel<T, false>, smem);
+    else
+        e = allow_smem(panel_update_kernel<T, false>, smem);
     double fl, by;
     trace_counts(G, level, p, kt, nodes, true, ccount, sizeof(T), &fl, &by);
     TraceScope ts(K_PANEL_UPDATE, fl, by, s);
     if (e == cudaSuccess) {
-        dim3 grid((unsigned)nodes, (unsigned)ceil_div(ccount, 32));
-        panel_update_kernel<T><<<grid, kThreads, smem, s>>>(G, A, Tws, level, p, kt, C, ldc, cfirst,
-                                                            ccount, trans);
+        // several 32-column blocks per CTA (V and T staged once) while keeping
+        // >= ~4 CTAs per SM of work
+        const int64_t nblk = ceil_div(ccount, 32);
+        const int64_t cpb = std::max<int64_t>(1, std::min<int64_t>(8, nodes * nblk / (4 * num_sms())));
+        dim3 grid((unsigned)nodes, (unsigned)ceil_div(nblk, cpb));
+        if (use_mma) {
+            if constexpr (sizeof(T) == 4)
+                panel_update_kernel<T, true><<<grid, kThreads, smem, s>>>(G, A, Tws, level, p, kt, C, ldc,
+                                                                          cfirst, ccount, trans, (int)cpb);
+        } else {
+            panel_update_kernel<T, false><<<grid, kThreads, smem, s>>>(G, A, Tws, level, p, kt, C, ldc,
+                                                                       cfirst, ccount, trans, (int)cpb);
+        }
         e = cudaGetLastError();
     }
     if (e != cudaSuccess) {
@@ -357,6 +372,38 @@ static int launch_fused(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, 
 
 // CAQR_FUSED=0 forces the split (one launch per level and panel) path; read
 // on every call so tests can compare both paths in one process.
+// CAQR_EARLY=0 disables the early-start overlap of the CAQR panel loop.
+static inline bool early_start_policy() {
+    const char* e = getenv("CAQR_EARLY");
+    return !(e && e[0] == '0');
+}
+// One non-blocking side stream and two timing-free events per device, created
+// on first use (the only resources the library ever creates).
+static bool side_stream(cudaStream_t* s2, cudaEvent_t* ev_ready, cudaEvent_t* ev_done) {
+    static std::mutex mu;
+    static cudaStream_t streams[64] = {};
+    static cudaEvent_t evs[64][2] = {};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev >= 64) return false;
+    std::lock_guard<std::mutex> lk(mu);
+    if (!streams[dev]) {
+        if (cudaStreamCreateWithFlags(&streams[dev], cudaStreamNonBlocking) != cudaSuccess) return false;
+        if (cudaEventCreateWithFlags(&evs[dev][0], cudaEventDisableTiming) != cudaSuccess ||
+            cudaEventCreateWithFlags(&evs[dev][1], cudaEventDisableTiming) != cudaSuccess)
+            return false;
+    }
+    *s2 = streams[dev];
+    *ev_ready = evs[dev][0];
+    *ev_done = evs[dev][1];
+    return true;
+}
+
+// CAQR_MMA=0 keeps the CAQR trailing update on FFMA (exact fp32 products).
+static inline bool mma_policy() {
+    const char* e = getenv("CAQR_MMA");
+    return !(e && e[0] == '0');
+}
+
 static inline int skinny_policy() {
     const char* e = getenv("CAQR_SKINNY");
     return (e && e[0] == '0') ? 0 : 1;
@@ -446,27 +493,28 @@ static int factor_group(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, 
 // order 0..npan-1; Q_g is the reverse.
 template <typename T>
 static int apply_group(const Geom& G, const T* A, const T* Tws, bool do_leaves, T* C,
-                       int64_t ldc, int64_t cfirst, int64_t ccount, int trans, cudaStream_t s) {
+                       int64_t ldc, int64_t cfirst, int64_t ccount, int trans, cudaStream_t s,
+                       bool mma = false) {
     int rc = 0;
     const int nl = tree_levels(G.P);
     if (trans) {
         if (do_leaves)
             for (int kt = 0; kt < G.K && !rc; ++kt)
                 for (int p = 0; p < G.npan && !rc; ++p)
-                    rc = launch_update<T>(G, A, Tws, -1, p, kt, G.P, C, ldc, cfirst, ccount, 1, s);
+                    rc = launch_update<T>(G, A, Tws, -1, p, kt, G.P, C, ldc, cfirst, ccount, 1, s, mma);
         for (int lv = 0; lv < nl && !rc; ++lv)
             for (int p = 0; p < G.npan && !rc; ++p)
                 rc = launch_update<T>(G, A, Tws, lv, p, 0, merges_at(G.P, lv), C, ldc, cfirst, ccount,
-                                      1, s);
+                                      1, s, mma);
     } else {
         for (int lv = nl - 1; lv >= 0 && !rc; --lv)
             for (int p = G.npan - 1; p >= 0 && !rc; --p)
                 rc = launch_update<T>(G, A, Tws, lv, p, 0, merges_at(G.P, lv), C, ldc, cfirst, ccount,
-                                      0, s);
+                                      0, s, mma);
         if (do_leaves)
             for (int kt = (int)G.K - 1; kt >= 0 && !rc; --kt)
                 for (int p = G.npan - 1; p >= 0 && !rc; --p)
-                    rc = launch_update<T>(G, A, Tws, -1, p, kt, G.P, C, ldc, cfirst, ccount, 0, s);
+                    rc = launch_update<T>(G, A, Tws, -1, p, kt, G.P, C, ldc, cfirst, ccount, 0, s, mma);
     }
     return rc;
 }
@@ -502,16 +550,48 @@ static int factor_impl(int64_t m, int64_t n, T* A, int64_t lda, T* R, int64_t ld
     if (!R) return -5;
     if (!ws) return -7;
     if (ws_bytes < plan_ws_bytes(pl)) return -8;
-    char* wsb = static_cast<char*>(ws);
+    // Group offsets in the workspace.
+    auto group_ptrs = [&](int64_t g, T** tws, int** sync) {
+        char* wsb = static_cast<char*>(ws);
+        for (int64_t q = 0; q < g; ++q) wsb += group_ws_bytes(group_geom(pl, q, lda), sizeof(T));
+        *tws = reinterpret_cast<T*>(wsb);
+        *sync = reinterpret_cast<int*>(wsb + group_t_bytes(group_geom(pl, g, lda), sizeof(T)));
+    };
+    // CAQR with early start ("the trailing matrix update can begin
+    // before the entire panel is factored"): after group g's TSQR, its Q^T is
+    // applied first to the next group's columns; the next TSQR then runs on a
+    // side stream while the rest of the trailing matrix is updated on `s`.
+    cudaStream_t s2 = nullptr;
+    cudaEvent_t ev_ready = nullptr, ev_done = nullptr;
+    const bool overlap = pl.ngroups > 1 && early_start_policy() && side_stream(&s2, &ev_ready, &ev_done);
     for (int64_t g = 0; g < pl.ngroups && !rc; ++g) {
         const Geom G = group_geom(pl, g, lda);
-        T* Tws = reinterpret_cast<T*>(wsb);
-        int* sync = reinterpret_cast<int*>(wsb + group_t_bytes(G, sizeof(T)));
-        rc = factor_group<T>(G, A, Tws, sync, true, s);
+        T* Tws;
+        int* sync;
+        group_ptrs(g, &Tws, &sync);
+        if (!overlap || g == 0) {
+            rc = factor_group<T>(G, A, Tws, sync, true, s);
+        } else if (cudaStreamWaitEvent(s, ev_done, 0) != cudaSuccess) {  // TSQR_g ran on s2
+            rc = CAQR_ERR_CUDA;
+        }
         const int64_t trail0 = G.col0 + G.ncols;
-        if (!rc && trail0 < n)  // CAQR trailing update
-            rc = apply_group<T>(G, A, Tws, true, A, lda, trail0, n - trail0, 1, s);
-        wsb += group_ws_bytes(G, sizeof(T));
+        if (rc || trail0 >= n) continue;
+        // CAQR trailing update; fp32: tensor cores (3xTF32)
+        const int64_t next_cols = overlap ? std::min<int64_t>(pl.nb, n - trail0) : n - trail0;
+        rc = apply_group<T>(G, A, Tws, true, A, lda, trail0, next_cols, 1, s, mma_policy());
+        if (!rc && overlap && g + 1 < pl.ngroups) {
+            const Geom Gn = group_geom(pl, g + 1, lda);
+            T* Twn;
+            int* syncn;
+            group_ptrs(g + 1, &Twn, &syncn);
+            if (cudaEventRecord(ev_ready, s) != cudaSuccess || cudaStreamWaitEvent(s2, ev_ready, 0) != cudaSuccess)
+                rc = CAQR_ERR_CUDA;
+            if (!rc) rc = factor_group<T>(Gn, A, Twn, syncn, true, s2);
+            if (!rc && cudaEventRecord(ev_done, s2) != cudaSuccess) rc = CAQR_ERR_CUDA;
+        }
+        if (!rc && next_cols < n - trail0)
+            rc = apply_group<T>(G, A, Tws, true, A, lda, trail0 + next_cols, n - trail0 - next_cols, 1, s,
+                                mma_policy());
     }
     if (!rc) rc = launch_extract_r<T>(n, A, lda, R, ldr, s);
     return rc;

@@ -284,10 +284,6 @@ __device__ __forceinline__ void factor_panel_regs(T* P, int RGP, int RG, int wp,
 // A group of 256 threads (8 warps) that runs one device routine: the whole
 // CTA in the one-role kernel, or one of the two roles of the look-ahead
 // kernel (named barrier per role).  tid is the group-local thread index.
-struct Grp {
-    int tid;
-    int bar;  // 0: __syncthreads over the CTA; >0: bar.sync bar, 256
-};
 __device__ __forceinline__ void gsync(const Grp& g) {
     if (g.bar == 0)
         __syncthreads();
@@ -637,6 +633,12 @@ __device__ __forceinline__ void mma_3xtf32(float (&d)[4], const uint32_t (&ah)[4
 
 // W(32 x 32) = V^T C on tensor cores; same warp split and deterministic
 // 4-way reduction as gemm_vtc.
+template <bool PAD = true>
+__device__ __forceinline__ int rowmap(int r) {
+    return PAD ? padr<float>(r) : r;
+}
+
+template <bool PAD>
 __device__ __forceinline__ void gemm_vtc_mma(const Grp& G, const float* Vs, const float* Cs, int RGP, int R32,
                                              float* Wp, float* W) {
     const int warp = G.tid >> 5, lane = G.tid & 31;
@@ -652,7 +654,7 @@ __device__ __forceinline__ void gemm_vtc_mma(const Grp& G, const float* Vs, cons
 #pragma unroll
             for (int e = 0; e < 4; ++e) acc[a][b][e] = 0.f;
     for (int k0 = rbeg; k0 < rend; k0 += 8) {
-        const int p0 = padr<float>(k0 + t), p1 = padr<float>(k0 + t + 4);
+        const int p0 = rowmap<PAD>(k0 + t), p1 = rowmap<PAD>(k0 + t + 4);
         uint32_t ah[2][4], al[2][4], bh[2][2], bl[2][2];
 #pragma unroll
         for (int mt = 0; mt < 2; ++mt) {
@@ -699,6 +701,7 @@ __device__ __forceinline__ void gemm_vtc_mma(const Grp& G, const float* Vs, cons
 
 // Cs(R32 x 32) <- Cs - V W2 on tensor cores (W2 in W, rows jj).  Warp w owns
 // row tiles {w, w + 8, ...} of 16 rows and all 4 column tiles.
+template <bool PAD>
 __device__ __forceinline__ void gemm2_mma(const Grp& G, const float* Vs, float* Cs, const float* W, int RGP,
                                           int R32) {
     const int warp = G.tid >> 5, lane = G.tid & 31;
@@ -714,7 +717,7 @@ __device__ __forceinline__ void gemm2_mma(const Grp& G, const float* Vs, float* 
         }
     for (int mt = warp; mt < R32 / 16; mt += kWarps) {
         const int m0 = 16 * mt;
-        const int r0 = padr<float>(m0 + g), r8 = padr<float>(m0 + g + 8);
+        const int r0 = rowmap<PAD>(m0 + g), r8 = rowmap<PAD>(m0 + g + 8);
         float d[4][4];
 #pragma unroll
         for (int nt = 0; nt < 4; ++nt) {
@@ -789,7 +792,7 @@ __device__ __forceinline__ void apply_block(const Grp& G, const T* Vs, const T* 
     for (int q = 0; q < 4; ++q) W[((tid >> 5) + 8 * q) * kTS + (tid & 31)] = w2[q];
     gsync(G);
     if constexpr (sizeof(T) == 4) {
-        gemm2_mma(G, Vs, const_cast<T*>(Cs), W, RGP, R32);
+        gemm2_mma<true>(G, Vs, const_cast<T*>(Cs), W, RGP, R32);
     } else {
     const int nq = R32 / 4;
     for (int u = tid; u < nq * 4; u += kThreads) {
@@ -1022,7 +1025,7 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
                 __syncthreads();
                 CAQR_PROF(6);
                 if constexpr (sizeof(T) == 4)
-                    gemm_vtc_mma(G0, P, Cs, RGP, R32, Wp, W);
+                    gemm_vtc_mma<true>(G0, P, Cs, RGP, R32, Wp, W);
                 else
                     gemm_vtc(G0, P, Cs, RGP, R32, Wp, W);
                 CAQR_PROF(7);
@@ -1114,7 +1117,7 @@ __device__ __forceinline__ void la_update_block(const Grp& GU, const Geom& g, T*
     stage_cols(GU, Cs, RGP, R32, static_cast<const T*>(A), g.lda, cb0, ncb, nr, RG, false, p);
     gsync(GU);
     if constexpr (sizeof(T) == 4)
-        gemm_vtc_mma(GU, P, Cs, RGP, R32, Wp, WU);
+        gemm_vtc_mma<true>(GU, P, Cs, RGP, R32, Wp, WU);
     else
         gemm_vtc(GU, P, Cs, RGP, R32, Wp, WU);
     apply_block(GU, P, Cs, Tt, WU, RGP, R32, RG, wp, 1, nr, A, g.lda, cb0, ncb);

@@ -304,10 +304,22 @@ __device__ __forceinline__ T vget(const double2& v, int i) {
     return i == 0 ? v.x : v.y;
 }
 
-template <typename T>
+// The mma (3xTF32 tensor-core) version of the two GEMMs, for the factor
+// path's CAQR trailing update only (apply_qt / apply_q / form_q use FFMA).
+struct Grp {
+    int tid;
+    int bar;  // 0: __syncthreads over the CTA; >0: bar.sync bar, 256
+};
+template <bool PAD>
+__device__ void gemm_vtc_mma(const Grp& G, const float* Vs, const float* Cs, int RGP, int R32, float* Wp,
+                             float* W);
+template <bool PAD>
+__device__ void gemm2_mma(const Grp& G, const float* Vs, float* Cs, const float* W, int RGP, int R32);
+
+template <typename T, bool MMA = false>
 __global__ void __launch_bounds__(kThreads)
 panel_update_kernel(Geom g, const T* A, const T* __restrict__ Tws, int level, int p, int kt, T* C,
-                    int64_t ldc, int64_t cfirst, int64_t ccount, int trans) {
+                    int64_t ldc, int64_t cfirst, int64_t ccount, int trans, int cpb) {
     using V4 = typename Vec4<T>::type;
     constexpr int VN = Vec4<T>::n;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -318,8 +330,6 @@ panel_update_kernel(Geom g, const T* A, const T* __restrict__ Tws, int level, in
     if (RG == 0) return;
     const int R32 = (RG + 31) & ~31;
     const int RGP = smem_col_stride<T>(RG);
-    const int64_t cb0 = cfirst + 32 * (int64_t)blockIdx.y;
-    const int ncb = (int)(cfirst + ccount - cb0 < 32 ? cfirst + ccount - cb0 : 32);
     T* Vs = reinterpret_cast<T*>(smem_raw);
     T* Cs = Vs + 32 * (size_t)RGP;
     T* Wp = Cs + 32 * (size_t)RGP;  // 4 x 32 x kTS
@@ -328,25 +338,52 @@ panel_update_kernel(Geom g, const T* A, const T* __restrict__ Tws, int level, in
     const int64_t c0 = g.col0 + 32 * p;
 
     // ---- stage V (implicit unit heads, structure masks) and C ---------------
-    for (int jj = warp; jj < 32; jj += kWarps) {
-        T* vs = Vs + (size_t)jj * RGP;
-        T* cs = Cs + (size_t)jj * RGP;
-        const T* acol = A + (c0 + jj) * g.lda;
-        const T* ccol = C + (cb0 + jj) * ldc;
-        for (int r = lane; r < R32; r += 32) {
-            T v = T(0), cv = T(0);
-            if (r < RG) {
-                if (jj < wp) {
-                    const bool st = panel_entry_stored(nr, r, jj, p) && (r >= nr.n0 || !nr.seg0_tri) &&
-                                    !(r < nr.n0 && r <= jj);
-                    v = v_entry<T>(nr, r, jj, p, st ? acol[gathered_row(nr, r)] : T(0));
+    // Each thread issues its loads in batches (4 columns x up to 9 row groups)
+    // before storing: one outstanding load per element would serialize the
+    // L2/HBM latency.
+    int64_t cb0 = 0;
+    int ncb = 0;
+    auto stage = [&](int pass) {
+        T buf[4][9];
+#pragma unroll
+        for (int a = 0; a < 4; ++a) {
+            const int jj = warp + kWarps * a;
+            const T* acol = A + (c0 + jj) * g.lda;
+            const T* ccol = C + (cb0 + jj) * ldc;
+#pragma unroll
+            for (int i = 0; i < 9; ++i) {
+                const int r = lane + 32 * i;
+                T val = T(0);
+                if (r < RG) {
+                    if (pass == 0) {
+                        if (jj < wp) {
+                            const bool st = panel_entry_stored(nr, r, jj, p) && (r >= nr.n0 || !nr.seg0_tri) &&
+                                            !(r < nr.n0 && r <= jj);
+                            val = st ? acol[gathered_row(nr, r)] : T(0);
+                        }
+                    } else if (jj < ncb) {
+                        val = ccol[gathered_row(nr, r)];
+                    }
                 }
-                if (jj < ncb) cv = ccol[gathered_row(nr, r)];
+                buf[a][i] = val;
             }
-            vs[r] = v;
-            cs[r] = cv;
         }
-    }
+#pragma unroll
+        for (int a = 0; a < 4; ++a) {
+            const int jj = warp + kWarps * a;
+            T* dst = (pass == 0 ? Vs : Cs) + (size_t)jj * RGP;
+#pragma unroll
+            for (int i = 0; i < 9; ++i) {
+                const int r = lane + 32 * i;
+                if (r < R32) {
+                    T val = buf[a][i];
+                    if (pass == 0) val = (r < RG && jj < wp) ? v_entry<T>(nr, r, jj, p, val) : T(0);
+                    dst[r] = val;
+                }
+            }
+        }
+    };
+    stage(0);  // V once per CTA
     {
         const T* tb = Tws + nr.tblk * (kPW * kPW);
         // only the wp x wp part of a T block is meaningful (the skinny kernel
@@ -354,8 +391,18 @@ panel_update_kernel(Geom g, const T* A, const T* __restrict__ Tws, int level, in
         for (int e = tid; e < kPW * kPW; e += kThreads)
             Tt[(e & 31) * kTS + (e >> 5)] = ((e & 31) < wp && (e >> 5) < wp) ? tb[e] : T(0);
     }
+    const int64_t nblk = (ccount + 31) / 32;
+    const int64_t blk_end = min(nblk, (int64_t)(blockIdx.y + 1) * cpb);
+    for (int64_t blk = (int64_t)blockIdx.y * cpb; blk < blk_end; ++blk) {
+    cb0 = cfirst + 32 * blk;
+    ncb = (int)(cfirst + ccount - cb0 < 32 ? cfirst + ccount - cb0 : 32);
+    __syncthreads();  // the previous block's readers of Cs are done
+    stage(1);
     __syncthreads();
 
+    if constexpr (MMA) {
+        gemm_vtc_mma<false>(Grp{tid, 0}, Vs, Cs, RGP, R32, Wp, W);
+    } else {
     // ---- W = V^T C : 4-way split over rows x 2 column halves per warp -------
     {
         const int ks = warp & 3, ch = warp >> 2;
@@ -400,20 +447,28 @@ panel_update_kernel(Geom g, const T* A, const T* __restrict__ Tws, int level, in
         W[jj * kTS + c] = s;
     }
     __syncthreads();
+    }
     // ---- W2 = T^T W (Q^T) or T W (Q); T upper triangular (Tt[r][c] = T[r][c])
+    // thread (column c, rows jj = jg + 8q); unrolled, T's zeros need no bounds
     T w2[4];
     {
+        const int c = tid & 31, jg = tid >> 5;
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
-            const int e = tid + q * kThreads;
-            const int jj = e >> 5, c = e & 31;
-            T s = T(0);
-            if (trans) {
-                for (int k = 0; k <= jj; ++k) s = fma(Tt[k * kTS + jj], W[k * kTS + c], s);
-            } else {
-                for (int k = jj; k < 32; ++k) s = fma(Tt[jj * kTS + k], W[k * kTS + c], s);
+        for (int q = 0; q < 4; ++q) w2[q] = T(0);
+#pragma unroll
+        for (int h = 0; h < 32; h += 8) {
+            T wc[8];
+#pragma unroll
+            for (int k2 = 0; k2 < 8; ++k2) wc[k2] = W[(h + k2) * kTS + c];
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const int jj = jg + 8 * q;
+                T acc = T(0);
+#pragma unroll
+                for (int k2 = 0; k2 < 8; ++k2)
+                    acc = fma(trans ? Tt[(h + k2) * kTS + jj] : Tt[jj * kTS + h + k2], wc[k2], acc);
+                w2[q] += acc;
             }
-            w2[q] = s;
         }
     }
     __syncthreads();
@@ -424,6 +479,15 @@ panel_update_kernel(Geom g, const T* A, const T* __restrict__ Tws, int level, in
     }
     __syncthreads();
 
+    if constexpr (MMA) {
+        gemm2_mma<false>(Grp{tid, 0}, Vs, Cs, W, RGP, R32);
+        __syncthreads();
+        for (int c = warp; c < ncb; c += kWarps) {
+            T* ccol = C + (cb0 + c) * ldc;
+            const T* cs = Cs + (size_t)c * RGP;
+            for (int r = lane; r < RG; r += 32) ccol[gathered_row(nr, r)] = cs[r];
+        }
+    } else {
     // ---- C -= V W2 : thread = (4 consecutive rows, 8 consecutive columns) ---
     const int nq = R32 / 4;
     for (int u = tid; u < nq * 4; u += kThreads) {
@@ -458,6 +522,8 @@ panel_update_kernel(Geom g, const T* A, const T* __restrict__ Tws, int level, in
                 if (r + i < RG) ccol[gathered_row(nr, r + i)] = acc[i][c];
         }
     }
+    }
+    }  // column blocks of this CTA
 }
 
 template <typename T>
