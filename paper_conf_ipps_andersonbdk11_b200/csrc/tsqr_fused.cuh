@@ -18,15 +18,16 @@
 
 namespace caqr {
 
-// Padded column layout of shared tiles, matched to the panel's thread layout
-// (PanelLayout<8>): rows 0..31 plain, then 28-row segments each followed by
-// PADS elements of padding, so the 8 segment owners of a column -- and 16-byte
-// vector loads by lanes at the same offset of different segments -- hit 8
-// different 16-byte bank groups (segment stride = 16 bytes mod 128).
+// Row index of a shared panel / C tile.  Plain (identity): every access pattern
+// that remains is conflict-free without row padding -- WB4 and the staging /
+// write-back loops have lanes on consecutive rows, and the GEMM fragments
+// differ by column, which the column stride (16 bytes mod 128) spreads over
+// the banks.  (An earlier 8-threads-per-column panel layout needed padding
+// after every 28-row segment; its integer divide cost ~8 % of the kernel's
+// instructions.)
 template <typename T>
 __host__ __device__ __forceinline__ int padr(int r) {
-    constexpr int PADS = sizeof(T) == 4 ? 8 : 6;
-    return r < 32 ? r : r + PADS * ((r - 32) / 28);
+    return r;
 }
 // Column stride for tiles of up to `rows` rows: (stride * sizeof(T)) % 128 == 16.
 template <typename T>
