@@ -311,10 +311,11 @@ struct Grp {
     int bar;  // 0: __syncthreads over the CTA; >0: bar.sync bar, 256
 };
 template <bool PAD>
-__device__ void gemm_vtc_mma(const Grp& G, const float* Vs, const float* Cs, int RGP, int R32, float* Wp,
-                             float* W);
+__device__ __forceinline__ void gemm_vtc_mma(const Grp& G, const float* Vs, const float* Cs, int RGP, int R32,
+                                             float* Wp, float* W);
 template <bool PAD>
-__device__ void gemm2_mma(const Grp& G, const float* Vs, float* Cs, const float* W, int RGP, int R32);
+__device__ __forceinline__ void gemm2_mma(const Grp& G, const float* Vs, float* Cs, const float* W, int RGP,
+                                          int R32);
 
 template <typename T, bool MMA = false>
 __global__ void __launch_bounds__(kThreads)
