@@ -334,7 +334,8 @@ __device__ __forceinline__ void warp_reduce_many(T (&v)[N], T* scr) {
 // ---------------------------------------------------------------------------
 template <typename T>
 __device__ __forceinline__ void factor_panel_wb4(const Grp& G, T* P, int RGP, int RG, int wp, T* tau_s, T* Tb,
-                                                 T* scr_all) {
+                                                 T* scr_all, const NodeRows* out_nr = nullptr, T* out_A = nullptr,
+                                                 int64_t out_lda = 0, int64_t out_c0 = 0, int out_p = 0) {
     const int warp = G.tid >> 5, lane = G.tid & 31;
     // block blk = 7 - warp: the warp that owns the next block always has the
     // highest warp id among the warps still applying the current one, so the
@@ -513,11 +514,29 @@ __device__ __forceinline__ void factor_panel_wb4(const Grp& G, T* P, int RGP, in
         }
     }
     gsync(G);  // every block applied: P's v columns are no longer read
+    if (out_A) {
+        // epilogue straight from registers: the stored form (R / v, structure
+        // masks) to global, the V form (unit head, zeros elsewhere) into P,
+        // zero columns beyond wp -- no extra pass over P
+        const NodeRows& nr = *out_nr;
 #pragma unroll
-    for (int q = 0; q < 4; ++q)
-        if (q < nc)
+        for (int q = 0; q < 4; ++q) {
+            T* col = out_A + (out_c0 + cb + q) * out_lda;
 #pragma unroll
-            for (int i = 0; i < 8; ++i) P[(size_t)(cb + q) * RGP + padr<T>(lane + 32 * i)] = x[q][i];
+            for (int i = 0; i < 8; ++i) {
+                const int r = lane + 32 * i;
+                const bool in = q < nc && r < RG;
+                if (in && panel_entry_stored(nr, r, cb + q, out_p)) col[gathered_row(nr, r)] = x[q][i];
+                P[(size_t)(cb + q) * RGP + padr<T>(r)] = in ? v_entry<T>(nr, r, cb + q, out_p, x[q][i]) : T(0);
+            }
+        }
+    } else {
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+            if (q < nc)
+#pragma unroll
+                for (int i = 0; i < 8; ++i) P[(size_t)(cb + q) * RGP + padr<T>(lane + 32 * i)] = x[q][i];
+    }
     gsync(G);
 }
 
@@ -980,32 +999,43 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
             const int R32 = (RG + 31) & ~31;
             const int64_t c0 = g.col0 + 32 * p;
             // ---- panel: stage, factor, store R/V, T ------------------------
-            stage_cols(G0, P, RGP, R32, A, g.lda, c0, wp, nr, RG, true, p);
-            if (threadIdx.x < 32) tau_s[threadIdx.x] = T(0);
-            __syncthreads();
-            CAQR_PROF(2);
-            factor_panel_wb4<T>(G0, P, RGP, RG, wp, tau_s, Wp, Cs);
-            CAQR_PROF(3);
-            {
+            if (level < 0 && p > 0) {
+                // The previous panel's LAST trailing block was this panel's
+                // columns over the previous node's gathered rows, still in Cs
+                // (updated).  A leaf's rows are those minus the first 32; a
+                // chain node's are the slot rows [32p, 32p+wp) (from global:
+                // not part of the previous node) and the same tile rows.
                 const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-                for (int jj = warp; jj < wp; jj += kWarps) {
-                    T* col = A + (c0 + jj) * g.lda;
+                const bool leaf = kt == 0;
+                T head[4];
+#pragma unroll
+                for (int a = 0; a < 4; ++a) {
+                    const int jj = warp + 8 * a;
+                    head[a] = (!leaf && lane < nr.n0 && jj < wp && panel_entry_stored(nr, lane, jj, p))
+                                  ? ldcg(A + (c0 + jj) * g.lda + gathered_row(nr, lane))
+                                  : T(0);
+                }
+#pragma unroll
+                for (int a = 0; a < 4; ++a) {
+                    const int jj = warp + 8 * a;
                     T* pc = P + (size_t)jj * RGP;
+                    const T* cc = Cs + (size_t)jj * RGP;
                     for (int r = lane; r < R32; r += 32) {
-                        const bool in = r < RG;
-                        const T val = pc[padr<T>(r)];
-                        if (in && panel_entry_stored(nr, r, jj, p)) col[gathered_row(nr, r)] = val;
-                        // V form in place: unit head, zeros above, structure masks
-                        const T v = in ? v_entry<T>(nr, r, jj, p, val) : T(0);
+                        T v;
+                        if (leaf) v = (r < RG && jj < wp) ? cc[padr<T>(r + 32)] : T(0);
+                        else if (r < nr.n0) v = head[a];
+                        else v = (r < RG && jj < wp) ? cc[padr<T>(r - nr.n0 + 32)] : T(0);
                         pc[padr<T>(r)] = v;
                     }
                 }
-                for (int jj = wp + warp; jj < 32; jj += kWarps) {
-                    T* pc = P + (size_t)jj * RGP;
-                    for (int r = lane; r < R32; r += 32) pc[padr<T>(r)] = T(0);
-                }
+            } else {
+                stage_cols(G0, P, RGP, R32, A, g.lda, c0, wp, nr, RG, true, p);
             }
+            if (threadIdx.x < 32) tau_s[threadIdx.x] = T(0);
             __syncthreads();
+            CAQR_PROF(2);
+            factor_panel_wb4<T>(G0, P, RGP, RG, wp, tau_s, Wp, Cs, &nr, A, g.lda, c0, p);
+            CAQR_PROF(3);
             CAQR_PROF(4);
             gemm_vtc(G0, P, P, RGP, R32, Wp, W);  // G = V^T V
             build_t(G0, W, tau_s, wp, Tt);
@@ -1019,8 +1049,12 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
             }
             CAQR_PROF(5);
             // ---- trailing columns of this node, 32 at a time -------------------
+            // (the block holding the NEXT panel's columns goes last, so that
+            // panel can be staged from Cs)
             const int64_t tfirst = c0 + 32, tend = g.col0 + g.ncols;
-            for (int64_t cb0 = tfirst; cb0 < tend; cb0 += 32) {
+            const int nblk = tend > tfirst ? (int)((tend - tfirst + 31) / 32) : 0;
+            for (int ib = 0; ib < nblk; ++ib) {
+                const int64_t cb0 = tfirst + 32 * ((ib + 1) % nblk);
                 const int ncb = (int)(tend - cb0 < 32 ? tend - cb0 : 32);
                 stage_cols(G0, Cs, RGP, R32, static_cast<const T*>(A), g.lda, cb0, ncb, nr, RG, false, p);
                 __syncthreads();
