@@ -356,19 +356,40 @@ __device__ __forceinline__ void factor_panel_wb4(const Grp& G, T* P, int RGP, in
     const int nblk = (wp + 3) / 4;
     for (int b = 0; b < nblk; ++b) {
         if (blk == b) {
+            // One 4-value warp reduction per reflector j = cb + q, taken on the
+            // UNSCALED column (rows r > j): its squared norm, its dots with the
+            // later columns k > q (v^T x_k = x_k[j] + scale * e_k) and with the
+            // earlier v_a, a < q (g_aq = v_a[j] + scale * f_a).  So the norm,
+            // the block update and the compact-WY Gram entries share one
+            // reduction instead of three.
             T tq[4] = {T(0), T(0), T(0), T(0)};
+            T gv[6] = {T(0), T(0), T(0), T(0), T(0), T(0)};
 #pragma unroll
             for (int q = 0; q < 4; ++q) {
                 if (q < nc) {
                     const int j = cb + q;
-                    T sg = T(0);
+                    T red[4] = {T(0), T(0), T(0), T(0)};
 #pragma unroll
                     for (int i = 0; i < 8; ++i) {
                         const int r = lane + 32 * i;
-                        sg = (r > j) ? fma(x[q][i], x[q][i], sg) : sg;
+                        const T xq = r > j ? x[q][i] : T(0);
+                        red[0] = fma(xq, xq, red[0]);
+#pragma unroll
+                        for (int m = 0; m < 3; ++m) {
+                            // slot 1 + m: e_{q+1+m} for m < 3 - q, else f_{m-(3-q)}
+                            const int k = m < 3 - q ? q + 1 + m : m - (3 - q);
+                            red[1 + m] = fma(xq, x[k][i], red[1 + m]);
+                        }
                     }
+                    warp_reduce_many<4>(red, scr);
                     const T al = __shfl_sync(0xffffffffu, x[q][0], j);
-                    sg = warp_sum(sg);
+                    T head[3];
+#pragma unroll
+                    for (int m = 0; m < 3; ++m) {
+                        const int k = m < 3 - q ? q + 1 + m : m - (3 - q);
+                        head[m] = __shfl_sync(0xffffffffu, x[k][0], j);
+                    }
+                    const T sg = red[0];
                     T tau = T(0), beta = al, scale = T(1);
                     if (j < RG && sg != T(0)) {
                         const T ss = fma(al, al, sg);
@@ -390,52 +411,21 @@ __device__ __forceinline__ void factor_panel_wb4(const Grp& G, T* P, int RGP, in
                         P[(size_t)j * RGP + padr<T>(r)] = v[i];
                     }
                     if (lane == 0) tau_s[j] = tau;
-                    // apply H_j to this warp's later columns (interleaved reductions)
-                    if (tau != T(0) && q + 1 < nc) {
-                        T d[4] = {T(0), T(0), T(0), T(0)};
 #pragma unroll
-                        for (int q2 = q + 1; q2 < 4; ++q2)
+                    for (int m = 0; m < 3; ++m) {
+                        if (m < 3 - q) {  // apply H_j to the later column k
+                            const int k = q + 1 + m;
+                            const T st = tau * fma(scale, red[1 + m], head[m]);
+                            if (tau != T(0))
 #pragma unroll
-                            for (int i = 0; i < 8; ++i) d[q2] = fma(v[i], x[q2][i], d[q2]);
-                        if (q == 0)
-                            warp_reduce_many<4>(d, scr);
-                        else
-#pragma unroll
-                            for (int o = 16; o > 0; o >>= 1)
-#pragma unroll
-                                for (int q2 = q + 1; q2 < 4; ++q2) d[q2] += __shfl_xor_sync(0xffffffffu, d[q2], o);
-#pragma unroll
-                        for (int q2 = q + 1; q2 < 4; ++q2) {
-                            const T st = tau * d[q2];
-#pragma unroll
-                            for (int i = 0; i < 8; ++i) x[q2][i] = fma(-st, v[i], x[q2][i]);
+                                for (int i = 0; i < 8; ++i) x[k][i] = fma(-st, v[i], x[k][i]);
+                        } else {  // Gram entry g_aq, a < q (index of (a, q), a < q)
+                            const int a = m - (3 - q);
+                            const int e = a == 0 ? q - 1 : (a == 1 ? q + 1 : 5);
+                            gv[e] = fma(scale, red[1 + m], head[m]);
                         }
                     }
                 }
-            }
-            // 4x4 compact-WY factor of the block: g_ab = v_a . v_b (a < b), then
-            // T[a][a] = tau_a, T[a][b] = -tau_b sum_{k=a}^{b-1} T[a][k] g_kb.
-            T gv[6];
-            {
-                T vv[4][8];
-#pragma unroll
-                for (int q = 0; q < 4; ++q)
-#pragma unroll
-                    for (int i = 0; i < 8; ++i) {
-                        const int r = lane + 32 * i, j = cb + q;
-                        vv[q][i] = (q < nc) ? (r > j ? x[q][i] : (r == j ? T(1) : T(0))) : T(0);
-                    }
-                int e = 0;
-#pragma unroll
-                for (int a = 0; a < 4; ++a)
-#pragma unroll
-                    for (int bb = a + 1; bb < 4; ++bb, ++e) {
-                        T g = T(0);
-#pragma unroll
-                        for (int i = 0; i < 8; ++i) g = fma(vv[a][i], vv[bb][i], g);
-                        gv[e] = g;
-                    }
-                warp_reduce_many<6>(gv, scr);
             }
             if (lane == 0) {
                 // gv index of (a, bb), a < bb: 0:(0,1) 1:(0,2) 2:(0,3) 3:(1,2) 4:(1,3) 5:(2,3)
