@@ -16,6 +16,7 @@
 #include "tsqr_fused.cuh"
 #include "tsqr_kernels.cuh"
 #include "tsqr_skinny.cuh"
+#include "tsqr_stream.cuh"
 
 namespace caqr {
 
@@ -59,6 +60,7 @@ constexpr int64_t kMaxGroup = 256;    // widest single TSQR panel group
 constexpr int64_t kMaxLeaf = 256;     // tallest tile the kernels stage in shared memory
 constexpr int64_t kFusedLeaf = 224;   // default tile height: [32 R rows; tile] fits 256 rows
 constexpr int64_t kChainTarget = 296; // chains per group (2 per B200 SM; device-independent constant)
+constexpr int64_t kStreamChains = 1184;  // skinny chains: 8 warps x 148 B200 SMs
 
 struct Plan {
     int64_t m = 0, n = 0;
@@ -86,7 +88,8 @@ static int make_plan(int64_t m, int64_t n, int dtype, const caqr_opts* o, int op
     // (only for genuinely tall inputs: below ~256k rows the block kernel's
     // fewer, larger tasks win, e.g. 4096 x 16: 0.13 ms vs 0.26 ms measured)
     pl->skinny = dtype == CAQR_F32 && n <= 16 && nb >= n && m >= (int64_t(1) << 18);
-    pl->chain_target = pl->skinny ? 2048 : kChainTarget;
+    // streaming kernel: one chain per warp, 8 warps per SM (148 SMs)
+    pl->chain_target = pl->skinny ? kStreamChains : kChainTarget;
     int64_t b = (o && o->leaf_rows > 0) ? o->leaf_rows
                                         : (pl->skinny ? (n <= 8 ? 256 : 128)
                                                       : (nb <= kFusedLeaf ? kFusedLeaf : kMaxLeaf));
@@ -404,9 +407,11 @@ static inline bool mma_policy() {
     return !(e && e[0] == '0');
 }
 
+// CAQR_SKINNY=0: no skinny kernel; =2: the older warp-per-task kernel with
+// flag-waiting merges instead of the streaming kernel.
 static inline int skinny_policy() {
     const char* e = getenv("CAQR_SKINNY");
-    return (e && e[0] == '0') ? 0 : 1;
+    return (e && e[0] == '0') ? 0 : (e && e[0] == '2') ? 2 : 1;
 }
 
 static inline int fused_policy() {
@@ -457,8 +462,70 @@ static int launch_skinny(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves,
     return 0;
 }
 
+// Streaming skinny TSQR (tsqr_stream.cuh): n <= 16, tiles of 256 (n <= 8) or
+// 128 rows, one chain per warp, 8 warps per CTA; true in *done if launched.
+template <typename T, int NC, int RPL, int NW = 8>
+static cudaError_t launch_stream_nc(const Geom& G, T* A, T* Tws, int* sync, bool vec, cudaStream_t s) {
+    const unsigned grid = (unsigned)ceil_div(G.P, NW);
+    const size_t smem = stream_smem_bytes<T, NC, RPL, NW>(grid);
+    const int nl = tree_levels(G.P);
+    cudaError_t e;
+    unsigned long long* prof = prof_buffer();
+    const char* dbe = getenv("CAQR_STREAM_DBG");
+    const int dbg = dbe ? atoi(dbe) : 0;
+    if (prof) cudaMemsetAsync(prof, 0xff, sizeof(unsigned long long), s);  // [0] is a running min
+    if (vec) {
+        e = allow_smem(tsqr_stream_kernel<T, NC, RPL, NW, true>, smem);
+        if (e == cudaSuccess)
+            tsqr_stream_kernel<T, NC, RPL, NW, true><<<grid, 32 * NW, smem, s>>>(G, A, Tws, sync, nl, prof, dbg);
+    } else {
+        e = allow_smem(tsqr_stream_kernel<T, NC, RPL, NW, false>, smem);
+        if (e == cudaSuccess)
+            tsqr_stream_kernel<T, NC, RPL, NW, false><<<grid, 32 * NW, smem, s>>>(G, A, Tws, sync, nl, prof, dbg);
+    }
+    return e == cudaSuccess ? cudaGetLastError() : e;
+}
+
+template <typename T>
+static int launch_stream(const Geom& G, T* A, T* Tws, int* sync, cudaStream_t s, bool* done) {
+    *done = false;
+    if constexpr (sizeof(T) == 4) {
+        const bool nc8 = G.ncols <= 8 && G.b == 256, nc16 = G.ncols <= 16 && G.b == 128;
+        if (!nc8 && !nc16) return 0;
+        // the CTAs' packed R's travel through the workspace's flag area
+        const int64_t nct = ceil_div(G.P, 8), nc = nc8 ? 8 : 16;
+        if ((int64_t)sizeof(T) * nct * nc * (nc + 1) / 2 > (int64_t)sizeof(int) * (G.L * G.npan - 32)) return 0;
+        if ((nc8 ? stream_smem_bytes<T, 8, 8, 8>(nct) : stream_smem_bytes<T, 16, 4, 8>(nct)) > 220 * 1024) return 0;
+        // 16-byte cp.async needs every tile column start 16-byte aligned
+        const bool vec = (reinterpret_cast<uintptr_t>(A) % 16 == 0) && (G.lda % 4 == 0) && (G.row0 % 4 == 0);
+        cudaError_t e = cudaMemsetAsync(sync, 0, group_sync_bytes(G), s);
+        if (e == cudaSuccess) {
+            double fl = 0, by = 0;
+            if (g_trace.on) {
+                const double mr = (double)G.mrows, nc = (double)G.ncols;
+                fl = 2.0 * mr * nc * nc - 2.0 / 3.0 * nc * nc * nc;
+                by = 2.0 * mr * nc * sizeof(T);
+            }
+            TraceScope ts(K_TSQR_SKINNY, fl, by, s);
+            e = nc8 ? launch_stream_nc<T, 8, 8>(G, A, Tws, sync, vec, s)
+                    : launch_stream_nc<T, 16, 4>(G, A, Tws, sync, vec, s);
+        }
+        if (e != cudaSuccess) {
+            g_last_cuda_error = (int)e;
+            return CAQR_ERR_CUDA;
+        }
+        *done = true;
+    }
+    return 0;
+}
+
 template <typename T>
 static int factor_group(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, cudaStream_t s) {
+    if (fused_policy() && do_leaves && G.npan == 1 && G.ncols <= 16 && skinny_policy() == 1) {
+        bool done = false;
+        const int rc = launch_stream<T>(G, A, Tws, sync, s, &done);
+        if (rc || done) return rc;
+    }
     if (fused_policy() && G.npan == 1 && G.ncols <= 16 && skinny_policy()) {
         bool done = false;
         const int rc = launch_skinny<T>(G, A, Tws, sync, do_leaves, s, &done);

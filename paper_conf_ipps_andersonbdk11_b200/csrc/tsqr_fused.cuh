@@ -340,7 +340,9 @@ __device__ __forceinline__ void factor_panel_wb4(const Grp& G, T* P, int RGP, in
     // block blk = 7 - warp: the warp that owns the next block always has the
     // highest warp id among the warps still applying the current one, so the
     // scheduler (highest-id-first) favours the critical path
-    const int blk = kWarps - 1 - warp;
+    // (through a shuffle so that the compiler knows blk -- and every branch on
+    // it around the warp reductions -- is warp-uniform: no WARPSYNC.COLLECTIVE)
+    const int blk = __shfl_sync(0xffffffffu, kWarps - 1 - warp, 0);
     const int cb = 4 * blk;
     const int nc = max(0, min(4, wp - cb));
     T* scr = scr_all + warp * (32 * 20 + 16);  // warp-private reduction scratch

@@ -1,0 +1,556 @@
+// tsqr_stream.cuh -- streaming TSQR of a skinny panel (n <= 16): one WARP per
+// chain, the chain's R resident in shared memory, tiles double-buffered by
+// cp.async, the binary tree climbed by the last-arriving warp.
+//
+// For the s-step Krylov shape ("millions of rows by less than ten
+// columns") the factorization is a stream of A through HBM: read each tile
+// once, write its Householder vectors once.  The plan and the implicit-Q
+// representation are the block kernels' (node_rows: chains of K tiles, P:L339-341
+// "any tree shape", then a binary tree over the chain R's), so
+// apply_qt / form_q replay it unchanged.  Per warp:
+//   * tile kt+1 is in flight (cp.async.cg, 16 B per lane per request when A is
+//     16-byte aligned) while tile kt is factored from registers;
+//   * the first tile is a leaf Householder QR ("factor"); every
+//     later one a structured QR of [R; tile] whose reflector heads sit in R
+//     (v_j = [e_j; y_j]), so R never leaves shared memory inside the chain;
+//   * per reflector ONE n-value warp all-reduce gives the squared norm, the dot
+//     products with the later columns (matvec of P:L704-711 on the unscaled
+//     column) and the Gram entries of the compact-WY T;
+//   * then the chain's R goes to its slot and the warp walks up the binary
+//     tree: at each merge an arrival counter picks the SECOND warp to arrive,
+//     which merges the two n x n triangles ("factor_tree") at once
+//     -- no warp ever spins on a flag.
+#pragma once
+#include "tsqr_fused.cuh"
+
+namespace caqr {
+
+__device__ __forceinline__ int64_t min64(int64_t a, int64_t b) { return a < b ? a : b; }
+
+// All N values summed over the warp; every lane gets all N totals.  Halving
+// butterfly (N/2 + N/4 + ... shuffles instead of 5 N), then the distinct
+// totals are broadcast through the warp's scratch.
+template <int N, typename T>
+__device__ __forceinline__ void warp_allreduce(T (&v)[N], T* scr) {
+    static_assert(N >= 1 && N <= 32 && (N & (N - 1)) == 0, "N: power of two <= 32");
+    const int lane = threadIdx.x & 31;
+    int idx = 0;
+#pragma unroll
+    for (int cnt = N, o = 16; cnt > 1; cnt >>= 1, o >>= 1) {
+        const bool up = (lane & o) != 0;
+#pragma unroll
+        for (int i = 0; i < cnt / 2; ++i) {
+            const T keep = up ? v[i + cnt / 2] : v[i];
+            const T send = up ? v[i] : v[i + cnt / 2];
+            v[i] = keep + __shfl_xor_sync(0xffffffffu, send, o);
+        }
+        idx += up ? cnt / 2 : 0;
+    }
+    constexpr int kDone = 32 / N;  // lanes [0, kDone) of each group hold one value index
+#pragma unroll
+    for (int o = kDone / 2; o >= 1; o >>= 1) v[0] += __shfl_xor_sync(0xffffffffu, v[0], o);
+    __syncwarp();
+    if ((lane & (kDone - 1)) == 0) scr[idx] = v[0];
+    __syncwarp();
+#pragma unroll
+    for (int i = 0; i < N; ++i) v[i] = scr[i];
+    __syncwarp();
+}
+
+// Householder scalars of one reflector (xLARFG, reading S1):
+// alpha = head, sg = squared tail norm.  tau = (beta-alpha)/beta,
+// scale = 1/(alpha-beta), beta = -copysign(sqrt(alpha^2 + sg), alpha);
+// sg == 0 (or no row) -> H = I.
+template <typename T>
+__device__ __forceinline__ void householder_scalars(T al, T sg, bool live, T& tau, T& beta, T& scale) {
+    tau = T(0);
+    beta = al;
+    scale = T(1);
+    if (live && sg != T(0)) {
+        const T ss = fma(al, al, sg);
+        const T aa = fabs(al);
+        T rmu, mu;
+        rsqrt_refined(ss, rmu, mu);
+        beta = -copysign(mu, al);
+        tau = fma(aa, rmu, T(1));
+        scale = copysign(rcp_refined(aa + mu), al);
+    }
+}
+
+// Per-warp shared state.
+template <typename T, int NC, int B>
+struct alignas(16) StreamWarp {
+    T buf[2][NC][B];   // double-buffered tile (column-major, B rows)
+    T R[NC][NC + 1];   // chain / subtree R, R[j][k] (upper)
+    T G[NC][NC + 1];   // Gram entries G[a][j] = v_a^T v_j (a < j)
+    T tau[NC];
+    T red[32];         // all-reduce scratch
+    T bc[2 * NC + 4];  // merge broadcast: v_j, tau, ...
+};
+
+// T (compact WY, xLARFT forward/columnwise) from tau and the Gram entries
+// G[a*ldg + j] = v_a^T v_j (a < j); column k of a group (k < NC, on) writes
+// row k into the 32x32 column-major slot tb (wp x wp used).
+template <typename T, int NC>
+__device__ __forceinline__ void stream_write_t(bool on, int k, const T* G, int ldg, const T* tau, int wp, T* tb,
+                                               int ldt = kPW) {
+    if (on && k < wp) {
+        T row[NC];
+#pragma unroll
+        for (int j = 0; j < NC; ++j) {
+            T acc = T(0);
+#pragma unroll
+            for (int q = 0; q < j; ++q) acc = fma(row[q], G[q * ldg + j], acc);  // row[q] == 0 for q < k
+            row[j] = (j == k) ? tau[j] : (j > k ? -tau[j] * acc : T(0));
+        }
+#pragma unroll
+        for (int j = 0; j < NC; ++j)
+            if (j < wp) tb[j * ldt + k] = row[j];
+    }
+}
+
+// cp.async of tile t (h rows, columns [c0, c0 + wp)) into buf (B rows x NC);
+// rows >= h and columns >= wp read as zeros.
+template <typename T, int NC, int B, bool VEC>
+__device__ __forceinline__ void stream_issue_tile(const Geom& g, const T* A, int64_t t, T (*buf)[B]) {
+    const int lane = threadIdx.x & 31;
+    const int64_t s = g.row0 + t * g.b;
+    const int h = (int)min64(g.b, g.mrows - t * g.b);
+    const int wp = g.ncols;
+    if constexpr (VEC) {
+        constexpr int E = 16 / sizeof(T);  // elements per 16-byte request
+#pragma unroll
+        for (int c = 0; c < NC; ++c) {
+#pragma unroll
+            for (int u = 0; u < B / (32 * E); ++u) {
+                const int r = E * (lane + 32 * u);
+                const int valid = c < wp ? max(0, min(E, h - r)) : 0;
+                const T* src = A + (g.col0 + min(c, wp - 1)) * g.lda + s + (valid > 0 ? r : 0);
+                const unsigned dst = (unsigned)__cvta_generic_to_shared(&buf[c][r]);
+                asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src),
+                             "r"(valid * (int)sizeof(T))
+                             : "memory");
+            }
+        }
+    } else {
+#pragma unroll
+        for (int c = 0; c < NC; ++c) {
+#pragma unroll
+            for (int u = 0; u < B / 32; ++u) {
+                const int r = lane + 32 * u;
+                const bool valid = c < wp && r < h;
+                const T* src = A + (g.col0 + min(c, wp - 1)) * g.lda + s + (valid ? r : 0);
+                const unsigned dst = (unsigned)__cvta_generic_to_shared(&buf[c][r]);
+                asm volatile("cp.async.ca.shared.global [%0], [%1], %2, %3;" ::"r"(dst), "l"(src),
+                             "n"((int)sizeof(T)), "r"(valid ? (int)sizeof(T) : 0)
+                             : "memory");
+            }
+        }
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+}
+
+// Leaf (kt == 0) or chain step (kt > 0) on the registers x[c][i] = row
+// lane + 32 i of column c.  Leaf: R ends in rows < NC of x (and is copied to
+// W.R); chain step: reflector heads in W.R, x becomes the dense V.
+template <typename T, int NC, int RPL, bool LEAF, int B>
+__device__ __forceinline__ void stream_tile_qr(T (&x)[NC][RPL], StreamWarp<T, NC, B>& W, int h) {
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int j = 0; j < NC; ++j) {
+        // slot 0: ||x_j||^2 ; slot 1+m (m < NC-1-j): x_j . x_{j+1+m} ; then x_a . x_j (a < j)
+        T red[NC];
+#pragma unroll
+        for (int q = 0; q < NC; ++q) red[q] = T(0);
+#pragma unroll
+        for (int i = 0; i < RPL; ++i) {
+            const T xj = (LEAF && i == 0 && lane <= j) ? T(0) : x[j][i];
+            red[0] = fma(xj, xj, red[0]);
+#pragma unroll
+            for (int q = 1; q < NC; ++q) {
+                const int k = q < NC - j ? j + q : q - (NC - j);  // later column, else earlier a
+                red[q] = fma(xj, x[k][i], red[q]);
+            }
+        }
+        // heads: leaf -- row j of every column (alpha, the later columns' heads,
+        // v_a[j] for a < j); chain step -- row j of R.  Read before the
+        // all-reduce (its __syncwarp orders them before lane 0 rewrites row j).
+        T hd[NC];
+#pragma unroll
+        for (int k = 0; k < NC; ++k) {
+            if constexpr (LEAF)
+                hd[k] = __shfl_sync(0xffffffffu, x[k][0], j);
+            else
+                hd[k] = k >= j ? W.R[j][k] : T(0);
+        }
+        warp_allreduce<NC>(red, W.red);
+        const T al = hd[j];
+        T tau, beta, scale;
+        householder_scalars(al, red[0], !LEAF || j < h, tau, beta, scale);
+        // later columns: s_k = head_k + scale * (x_j . x_k); x_k -= tau s_k v_j
+#pragma unroll
+        for (int q = 1; q < NC; ++q) {
+            if (q < NC - j) {
+                const int k = j + q;
+                const T head = hd[k];
+                const T sk = fma(scale, red[q], head);
+                const T f = tau * sk;
+                const T fs = f * scale;
+#pragma unroll
+                for (int i = 0; i < RPL; ++i) {
+                    if (LEAF && i == 0 && lane < j) continue;
+                    if (LEAF && i == 0 && lane == j)
+                        x[k][0] -= f;
+                    else
+                        x[k][i] = fma(-fs, x[j][i], x[k][i]);
+                }
+                if (!LEAF && lane == 0) W.R[j][k] = head - f;
+            } else if (lane == 0) {  // Gram entry (a, j), a < j
+                const int a = q - (NC - j);
+                W.G[a][j] = LEAF ? fma(scale, red[q], hd[a]) : scale * red[q];
+            }
+        }
+#pragma unroll
+        for (int i = 0; i < RPL; ++i) {
+            if (LEAF && i == 0 && lane < j) continue;
+            if (LEAF && i == 0 && lane == j)
+                x[j][0] = beta;
+            else
+                x[j][i] *= scale;
+        }
+        if (lane == 0) {
+            W.tau[j] = tau;
+            if (!LEAF) W.R[j][j] = beta;
+        }
+        __syncwarp();
+    }
+    if constexpr (LEAF) {  // R = rows < NC of the tile (upper part)
+        if (lane < NC)
+#pragma unroll
+            for (int k = 0; k < NC; ++k) W.R[lane][k] = k >= lane ? x[k][0] : T(0);
+        __syncwarp();
+    }
+}
+
+// Merge of two upper-triangular n x n factors [Ra; Rb] (Rb: nb rows) by a
+// GROUP of NC lanes, lane k of the group holding column k of both (R[i*ld+k]).
+// Reflector j: head Ra[j][j], tail Rb[0..j][j] (structured).
+// Out: Ro = new R (may alias Ra or Rb: inputs are read into registers
+// first), rb = V_2 column k (rows <= k), G / tau for T.  All lanes of the warp
+// call it (uniform __syncwarp); groups with on == false only synchronise.
+template <typename T, int NC>
+__device__ __forceinline__ void merge_group(bool on, int k, const T* Ra, const T* Rb, int ld, int nb, T* Ro,
+                                            T (&rb)[NC], T* G, int ldg, T* tau, T* bc) {
+    T ra[NC];
+#pragma unroll
+    for (int i = 0; i < NC; ++i) {
+        ra[i] = on ? Ra[i * ld + k] : T(0);
+        rb[i] = (on && i < nb && i <= k) ? Rb[i * ld + k] : T(0);
+    }
+    __syncwarp();
+#pragma unroll
+    for (int j = 0; j < NC; ++j) {
+        if (on && k == j) {
+            T s0 = T(0), s1 = T(0);
+#pragma unroll
+            for (int i = 0; i <= j; i += 2) {
+                s0 = fma(rb[i], rb[i], s0);
+                if (i + 1 <= j) s1 = fma(rb[i + 1], rb[i + 1], s1);
+            }
+            T tj, beta, scale;
+            householder_scalars(ra[j], s0 + s1, true, tj, beta, scale);
+            ra[j] = beta;
+#pragma unroll
+            for (int i = 0; i <= j; ++i) {
+                rb[i] *= scale;
+                bc[i] = rb[i];
+            }
+            bc[NC] = tj;
+            tau[j] = tj;
+        }
+        __syncwarp();
+        if (on) {
+            if (k > j) {
+                const T tj = bc[NC];
+                T s0 = ra[j], s1 = T(0);
+#pragma unroll
+                for (int i = 0; i <= j; i += 2) {
+                    s0 = fma(bc[i], rb[i], s0);
+                    if (i + 1 <= j) s1 = fma(bc[i + 1], rb[i + 1], s1);
+                }
+                const T f = tj * (s0 + s1);
+                ra[j] -= f;
+#pragma unroll
+                for (int i = 0; i <= j; ++i) rb[i] = fma(-f, bc[i], rb[i]);
+            } else if (k < j) {  // Gram entry (k, j): the R_a parts are unit vectors
+                T gsum = T(0);
+#pragma unroll
+                for (int i = 0; i <= j; ++i) gsum = fma(rb[i], bc[i], gsum);
+                G[k * ldg + j] = gsum;
+            }
+        }
+        __syncwarp();
+    }
+    if (on)
+#pragma unroll
+        for (int i = 0; i < NC; ++i) Ro[i * ld + k] = i <= k ? ra[i] : T(0);
+    __syncwarp();
+}
+
+// Shared memory of the last CTA's tree phase: every CTA's R (slot c * NW),
+// then per merge unit (a group of NC lanes) its G / tau / broadcast scratch.
+template <typename T, int NC>
+struct TreeUnit {
+    T G[NC][NC + 1];
+    T tau[NC];
+    T bc[NC + 4];
+};
+
+template <typename T, int NC, int RPL, int NW, bool VEC>
+__global__ void __launch_bounds__(32 * NW, 1)
+tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int nlevels,
+                   unsigned long long* prof, int dbg) {
+    static_assert((NW & (NW - 1)) == 0, "NW: power of two (in-CTA tree levels)");
+    constexpr int B = 32 * RPL;
+    constexpr int LDR = NC + 1;
+    using SW = StreamWarp<T, NC, B>;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ int s_last;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    SW* Ws = reinterpret_cast<SW*>(smem_raw);
+    SW& W = Ws[warp];
+    const int64_t base = (int64_t)blockIdx.x * NW;
+    const int64_t chain = base + warp;
+    // warp-uniform values through a shuffle: the compiler then knows the
+    // branches around the warp collectives are uniform (a thread-dependent
+    // condition compiles every shuffle to slow WARPSYNC.COLLECTIVE code)
+    const bool live = __shfl_sync(0xffffffffu, chain < g.P ? 1 : 0, 0) != 0;
+    const int wp = g.ncols;
+
+    // optional timestamps (diagnostics, CAQR_PROFILE=1): [0] min chain start,
+    // [1] max chain end, [2] root done (ns, globaltimer); [3] sum of chain
+    // times; [4] cycles waiting for tiles; [5] last-CTA tree time; [6] merges
+    auto gtime = []() {
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        return t;
+    };
+    const unsigned long long tstart = prof ? gtime() : 0ull;
+    unsigned long long twait = 0;
+    // slot rows of tree leaf sl (top rows of its chain's first tile)
+    auto slot_ptr = [&](int64_t sl) { return A + g.col0 * g.lda + g.row0 + sl * g.bm; };
+    auto slot_h = [&](int64_t sl) { return min64(g.b, g.mrows - sl * g.bm); };
+    // V_2 of a merge into R_b's slot (upper incl. diagonal) and its T
+    auto store_merge = [&](bool on, int k, int64_t sb, const T (&rb)[NC], const T* G, const T* tau) {
+        const int64_t hb = slot_h(sb);
+        if (on && k < wp) {
+            T* bb = slot_ptr(sb) + k * g.lda;
+#pragma unroll
+            for (int i = 0; i < NC; ++i)
+                if (i <= k && i < hb) bb[i] = rb[i];
+        }
+        stream_write_t<T, NC>(on, k, G, LDR, tau, wp, Tws + ((g.L + sb * g.K) * g.npan) * (kPW * kPW));
+    };
+
+    // ---- the chain: tiles chain*K .., leaf first; R stays in W.R ----------
+    if (live) {
+        const int64_t t0 = chain * g.K;
+        const int ntile = __shfl_sync(0xffffffffu, (int)min64(g.K, g.L - t0), 0);
+        stream_issue_tile<T, NC, B, VEC>(g, A, t0, W.buf[0]);
+        for (int kt = 0; kt < ntile; ++kt) {
+            const int64_t t = t0 + kt;
+            const long long cw0 = prof ? clock64() : 0;
+            if (kt + 1 < ntile) {
+                stream_issue_tile<T, NC, B, VEC>(g, A, t + 1, W.buf[(kt + 1) & 1]);
+                asm volatile("cp.async.wait_group 1;" ::: "memory");
+            } else {
+                asm volatile("cp.async.wait_group 0;" ::: "memory");
+            }
+            if (prof) twait += clock64() - cw0;
+            __syncwarp();
+            const int h = (int)min64(g.b, g.mrows - t * g.b);
+            T x[NC][RPL];
+#pragma unroll
+            for (int c = 0; c < NC; ++c)
+#pragma unroll
+                for (int i = 0; i < RPL; ++i) x[c][i] = W.buf[kt & 1][c][lane + 32 * i];
+            __syncwarp();  // the buffer is refilled (tile kt + 2) after this point
+            if (kt == 0)
+                stream_tile_qr<T, NC, RPL, true, B>(x, W, h);
+            else
+                stream_tile_qr<T, NC, RPL, false, B>(x, W, h);
+            // V (and a leaf's R) back over the tile; T into its slot
+            const int64_t s = g.row0 + t * g.b;
+#pragma unroll
+            for (int c = 0; c < NC; ++c) {
+                if (c < wp) {
+                    T* col = A + (g.col0 + c) * g.lda + s;
+#pragma unroll
+                    for (int i = 0; i < RPL; ++i) {
+                        const int r = lane + 32 * i;
+                        if (r < h) col[r] = x[c][i];
+                    }
+                }
+            }
+            stream_write_t<T, NC>(lane < NC, lane, &W.G[0][0], LDR, W.tau, wp, Tws + (t * g.npan) * (kPW * kPW));
+            __syncwarp();
+        }
+        if (prof && lane == 0) {
+            const unsigned long long te = gtime();
+            atomicMin(prof + 0, tstart);
+            atomicMax(prof + 1, te);
+            atomicAdd(prof + 3, te - tstart);
+            atomicAdd(prof + 4, twait);
+        }
+    }
+
+    // ---- tree levels inside the CTA: warps' R's in shared memory ----------
+    int l = 0;
+    for (; (2 << l) <= NW && l < nlevels; ++l) {
+        __syncthreads();
+        const int hl = 1 << l;
+        const bool on = __shfl_sync(0xffffffffu, (live && (warp & (2 * hl - 1)) == 0 && chain + hl < g.P) ? 1 : 0, 0);
+        if (on) {  // warp-uniform
+            T rb[NC];
+            const int64_t sb = chain + hl;
+            merge_group<T, NC>(lane < NC, lane, &W.R[0][0], &Ws[warp + hl].R[0][0], LDR,
+                               (int)min64(NC, slot_h(sb)), &W.R[0][0], rb, &W.G[0][0], LDR, W.tau, W.bc);
+            store_merge(lane < NC, lane, sb, rb, &W.G[0][0], W.tau);
+        }
+    }
+    __syncthreads();
+    auto store_r = [&](const T* R, int64_t sl) {  // R (upper) into the slot's top rows
+        const int64_t hs = slot_h(sl);
+        if (lane < NC && lane < wp) {
+            T* col = slot_ptr(sl) + lane * g.lda;
+#pragma unroll
+            for (int i = 0; i < NC; ++i)
+                if (i <= lane && i < hs) col[i] = R[i * LDR + lane];
+        }
+    };
+    if (l >= nlevels) {  // the whole tree fitted in this CTA
+        if (warp == 0) store_r(&W.R[0][0], base);
+        return;
+    }
+    // the CTA's R (packed upper triangle, contiguous per CTA) into the
+    // workspace's exchange area -- one coalesced read for the last CTA
+    constexpr int NP = NC * (NC + 1) / 2;
+    T* Rx = reinterpret_cast<T*>(sync + 64);
+    if (warp == 0 && lane < NC)
+#pragma unroll
+        for (int i = 0; i < NC; ++i)
+            if (i <= lane) Rx[blockIdx.x * NP + lane * (lane + 1) / 2 + i] = W.R[i][lane];
+
+    // ---- the last CTA to get here climbs the rest of the tree ---------------
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) s_last = atomicAdd(sync + 32, 1) == (int)gridDim.x - 1;
+    __syncthreads();
+    if (!s_last) return;
+    __threadfence();
+    const unsigned long long tt0 = prof ? gtime() : 0ull;
+    const int nct = (int)gridDim.x;
+    T* Rall = reinterpret_cast<T*>(smem_raw);  // [nct][NC][LDR]
+    using TU = TreeUnit<T, NC>;
+    TU* units = reinterpret_cast<TU*>(Rall + (size_t)nct * NC * LDR);
+    // merges whose V_2 / T stay in shared memory until the tree is done
+    // (NC <= 8): the tree's few global stores then leave in one burst instead
+    // of one round trip per level behind the chains' write-back
+    constexpr bool DEFER = NC <= 8;
+    T* Vd = reinterpret_cast<T*>(units + NW * (32 / NC));  // [nct][NP]
+    T* Td = Vd + (size_t)nct * NP;                         // [nct][NC][NC]
+    {   // every CTA's R: independent coalesced loads in batches, then the stores
+        constexpr int BATCH = 8;
+        const int total = nct * NP;
+        for (int e0 = threadIdx.x; e0 < total; e0 += 32 * NW * BATCH) {
+            T v[BATCH];
+#pragma unroll
+            for (int u = 0; u < BATCH; ++u) {
+                const int e = e0 + u * 32 * NW;
+                v[u] = e < total ? __ldcg(Rx + e) : T(0);
+            }
+#pragma unroll
+            for (int u = 0; u < BATCH; ++u) {
+                const int e = e0 + u * 32 * NW;
+                if (e < total) {
+                    const int c = e / NP, q = e % NP;
+                    int kk = 0;
+                    while ((kk + 1) * (kk + 2) / 2 <= q) ++kk;
+                    const int i = q - kk * (kk + 1) / 2;
+                    Rall[(size_t)c * NC * LDR + i * LDR + kk] = v[u];
+                }
+            }
+        }
+        for (int e = threadIdx.x; e < nct * NC * NC; e += 32 * NW) {  // strict lower parts
+            const int c = e / (NC * NC), i = (e / NC) % NC, kk = e % NC;
+            if (i > kk) Rall[(size_t)c * NC * LDR + i * LDR + kk] = T(0);
+        }
+    }
+    if (prof && threadIdx.x == 0) prof[7] = gtime() - tt0;
+    const long long cl0 = clock64();
+    constexpr int GPW = 32 / NC;  // merge groups per warp
+    const int grp = lane / NC, k = lane % NC;
+    const int unit = warp * GPW + grp;
+    TU& U = units[unit];
+    for (; l < nlevels; ++l) {
+        __syncthreads();
+        const int64_t hl = int64_t(1) << l;
+        const int64_t nm = (g.P - 1 >= hl) ? (g.P - 1 - hl) / (2 * hl) + 1 : 0;
+        for (int64_t r0 = 0; r0 < nm; r0 += NW * GPW) {  // rounds of NW*GPW merges (warp-uniform loop)
+            const int64_t node = r0 + unit;
+            const bool on = node < nm;
+            const int64_t sa = node << (l + 1), sb = sa + hl;
+            const int ca = on ? (int)(sa / NW) : 0, cb = on ? (int)(sb / NW) : 0;
+            T rb[NC];
+            T* Ra = Rall + (size_t)ca * NC * LDR;
+            const long long c0 = clock64();
+            if (!(dbg & 2))
+            merge_group<T, NC>(on, k, Ra, Rall + (size_t)cb * NC * LDR, LDR,
+                               on ? (int)min64(NC, slot_h(sb)) : 0, Ra, rb, &U.G[0][0], LDR, U.tau, U.bc);
+            const long long c1 = clock64();
+            if (prof && threadIdx.x == 0) { prof[9] += c1 - c0; prof[12] += 1; }
+            if (dbg & 1) {
+            } else if (DEFER) {
+                if (on)
+#pragma unroll
+                    for (int i = 0; i < NC; ++i)
+                        if (i <= k) Vd[(size_t)cb * NP + k * (k + 1) / 2 + i] = rb[i];
+                stream_write_t<T, NC>(on, k, &U.G[0][0], LDR, U.tau, wp, Td + (size_t)cb * NC * NC, NC);
+                __syncwarp();
+                if (prof && threadIdx.x == 0) prof[10] += clock64() - c1;
+            } else {
+                store_merge(on, k, sb, rb, &U.G[0][0], U.tau);
+            }
+            if (prof && on && k == 0) atomicAdd(prof + 6, 1ull);
+        }
+    }
+    __syncthreads();
+    if (prof && threadIdx.x == 0) prof[11] = clock64() - cl0;
+    if (warp == 0) store_r(Rall, 0);  // the root R
+    if (DEFER && !(dbg & 1)) {  // V_2 into every R_b slot (CTA c >= 1), T blocks
+        for (int e = threadIdx.x; e < nct * NC * NC; e += 32 * NW) {
+            const int c = e / (NC * NC), j = (e / NC) % NC, kk = e % NC;  // T[kk][j] / V_2 (j, kk)
+            if (c == 0) continue;
+            const int64_t sb = (int64_t)c * NW;
+            if (j < wp && kk < wp)
+                Tws[((g.L + sb * g.K) * g.npan) * (kPW * kPW) + j * kPW + kk] = Td[(size_t)c * NC * NC + j * NC + kk];
+            if (j <= kk && kk < wp && j < slot_h(sb))
+                slot_ptr(sb)[kk * g.lda + j] = Vd[(size_t)c * NP + kk * (kk + 1) / 2 + j];
+        }
+    }
+    if (prof && threadIdx.x == 0) {
+        const unsigned long long te = gtime();
+        atomicAdd(prof + 5, te - tt0);
+        atomicMax(prof + 2, te);
+    }
+}
+
+template <typename T, int NC, int RPL, int NW>
+inline size_t stream_smem_bytes(int64_t nct) {
+    const size_t chain = sizeof(StreamWarp<T, NC, 32 * RPL>) * NW;
+    const size_t tree = sizeof(T) * (size_t)nct * NC * (NC + 1) + sizeof(TreeUnit<T, NC>) * NW * (32 / NC) +
+                        (NC <= 8 ? sizeof(T) * (size_t)nct * (NC * (NC + 1) / 2 + NC * NC) : 0);
+    return chain > tree ? chain : tree;
+}
+
+}  // namespace caqr

@@ -323,8 +323,8 @@ def test_lookahead_kernel(caqr, monkeypatch):
 
 @pytest.mark.parametrize("m,n", [(600_000, 16), (2_100_000, 8), (530_000, 3)])
 def test_skinny_chains(caqr, m, n):
-    """Skinny fp32 panels (n <= 16) go to the warp-per-task kernel; with more
-    tiles than its 2048-chain target the tiles form chains."""
+    """Skinny fp32 panels (n <= 16) go to the streaming warp-per-chain kernel;
+    with more tiles than its 1184-chain target the tiles form chains."""
     info = caqr.caqr_plan_info(m, n)
     assert info["chains"] < info["leaves"]
     A = workloads.gaussian(m, n, seed=n)
@@ -338,6 +338,46 @@ def test_skinny_vs_block_kernel(caqr, monkeypatch):
     monkeypatch.setenv("CAQR_SKINNY", "0")
     R2, _, _, _ = gpu_qr(caqr, A, want_q=False)
     assert np.linalg.norm(R1 - R2) / np.linalg.norm(R1) <= 1e-5
+
+
+@pytest.mark.parametrize("m,n,pad", [(300_001, 5, 1), (262_147, 9, 3), (400_000, 1, 0), (1_000_003, 16, 0),
+                                     (524_288, 8, 4)])
+def test_stream_kernel_layouts(caqr, m, n, pad):
+    """Streaming skinny kernel (tsqr_stream.cuh): ragged last tile, n = 1 / 5 /
+    8 / 9 / 16, lda = m + pad (pad % 4 != 0 -> 4-byte cp.async path) -- R
+    against the oracle, Q^T Q = I, A = QR, Q^T A = [R; 0] through apply_qt."""
+    bd = BOUNDS[np.float32]
+    A = workloads.gaussian(m, n, seed=m % 97 + n)
+    big = caqr.colmajor_empty(m + pad, n, torch.float32)
+    Av = big[:m]
+    Av.copy_(torch.from_numpy(A))
+    R, ws = caqr.caqr_factor(Av)
+    Q = caqr.caqr_form_q(Av, ws)
+    C = caqr.colmajor_empty(m, n, torch.float32)
+    C.copy_(torch.from_numpy(A))
+    caqr.caqr_apply_qt(Av, ws, C)
+    torch.cuda.synchronize()
+    R64, Q64 = R.cpu().double().numpy(), Q.cpu().double().numpy()
+    A64 = A.astype(np.float64)
+    Ro = oracle.normalize_signs(oracle.qr(A64, want_q=False))
+    assert np.linalg.norm(oracle.normalize_signs(R64) - Ro) / np.linalg.norm(Ro) <= bd["r"]
+    assert np.linalg.norm(A64 - Q64 @ R64) / np.linalg.norm(A64) <= bd["res"]
+    assert np.linalg.norm(Q64.T @ Q64 - np.eye(n)) <= bd["orth"]
+    top = C.cpu().double().numpy()
+    assert np.linalg.norm(top[:n] - R64) / np.linalg.norm(R64) <= bd["res"]
+    assert np.linalg.norm(top[n:]) / np.linalg.norm(R64) <= 10 * bd["res"]
+
+
+def test_stream_vs_warp_task_kernel(caqr, monkeypatch):
+    """Streaming kernel and the older flag-waiting warp-per-task kernel run the
+    same plan: R agrees to rounding, both against the oracle."""
+    A = workloads.gaussian(2_000_000, 8, seed=4)
+    R1, _, _, _ = gpu_qr(caqr, A, want_q=False)
+    monkeypatch.setenv("CAQR_SKINNY", "2")
+    R2, _, _, _ = gpu_qr(caqr, A, want_q=False)
+    assert np.linalg.norm(R1 - R2) / np.linalg.norm(R1) <= 1e-5
+    Ro = oracle.normalize_signs(oracle.qr(A.astype(np.float64), want_q=False))
+    assert np.linalg.norm(oracle.normalize_signs(R1) - Ro) / np.linalg.norm(Ro) <= 1e-4
 
 
 @pytest.mark.parametrize("dtype", [np.float32, np.float64], ids=["f32", "f64"])
