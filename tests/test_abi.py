@@ -62,7 +62,7 @@ def test_plan_info(L):
     p = caqr.caqr_plan_info(4096, 16, 0, caqr.make_opts(leaf_rows=128))
     assert p["leaf_rows"] == 128 and p["leaves"] == 32 and p["tree_levels"] == 5
     p = caqr.caqr_plan_info(4_000_000, 8)  # skinny: 256-row tiles, ~2048 chains
-    assert p["leaf_rows"] == 256 and p["leaves"] == 15625 and p["chains"] == 1954 and p["launches"] == 2
+    assert p["leaf_rows"] == 256 and p["leaves"] == 15625 and p["chains"] == 1117 and p["launches"] == 2
 
 
 def test_info_codes_without_gpu(L):
