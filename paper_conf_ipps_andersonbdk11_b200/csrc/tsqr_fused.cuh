@@ -625,7 +625,11 @@ __device__ __forceinline__ void split_tf32(float x, uint32_t& hi, uint32_t& lo) 
     uint32_t h, l;
     asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(h) : "f"(x));
     const float r = x - __uint_as_float(h);
+#ifdef CAQR_CHEAP_SPLIT
+    l = __float_as_uint(r);
+#else
     asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(l) : "f"(r));
+#endif
     hi = h;
     lo = l;
 }
@@ -765,7 +769,7 @@ __device__ __forceinline__ void gemm2_mma(const Grp& G, const float* Vs, float* 
 template <typename T>
 __device__ __forceinline__ void apply_block(const Grp& G, const T* Vs, const T* Cs, const T* Tt, T* W, int RGP, int R32,
                                             int RG, int wp, int trans, const NodeRows& nr, T* C,
-                                            int64_t ldc, int64_t cb0, int ncb) {
+                                            int64_t ldc, int64_t cb0, int ncb, bool vec = false) {
     using V4 = typename Vec4<T>::type;
     constexpr int VN = Vec4<T>::n;
     const int tid = G.tid;
@@ -859,13 +863,77 @@ __device__ __forceinline__ void apply_block(const Grp& G, const T* Vs, const T* 
     gsync(G);
     {
         const int warp = tid >> 5, lane = tid & 31;
-        for (int c = warp; c < ncb; c += kWarps) {
-            T* ccol = C + (cb0 + c) * ldc;
-            const T* cs = Cs + (size_t)c * RGP;
-            for (int r = lane; r < RG; r += 32) ccol[gathered_row(nr, r)] = cs[padr<T>(r)];
+        if (sizeof(T) == 4 && vec) {  // float4 stores: rows 4q..4q+3 lie in one segment
+            for (int c = warp; c < ncb; c += kWarps) {
+                T* ccol = C + (cb0 + c) * ldc;
+                const T* cs = Cs + (size_t)c * RGP;
+                for (int r = 4 * lane; r < RG; r += 128) {
+                    if (r + 4 <= RG) {
+                        *reinterpret_cast<float4*>(ccol + gathered_row(nr, r)) =
+                            *reinterpret_cast<const float4*>(cs + r);
+                    } else {
+                        for (int q = r; q < RG; ++q) ccol[gathered_row(nr, q)] = cs[q];
+                    }
+                }
+            }
+        } else {
+            for (int c = warp; c < ncb; c += kWarps) {
+                T* ccol = C + (cb0 + c) * ldc;
+                const T* cs = Cs + (size_t)c * RGP;
+                for (int r = lane; r < RG; r += 32) ccol[gathered_row(nr, r)] = cs[padr<T>(r)];
+            }
         }
     }
     gsync(G);
+}
+
+// cp.async (LDGSTS) staging of a C block (gathered rows, ncol <= 32 columns
+// from col0) into S (column-major, stride RGP, rows [RG, R32) zero-filled):
+// no register round trip and, with vec, a quarter of the load instructions
+// and address arithmetic of stage_cols.  vec: 16-byte requests (A 16-byte
+// aligned, lda % 4 == 0, row segments starting on multiples of 4).  Caller
+// waits (cp.async.wait_group) and synchronises.
+__device__ __forceinline__ void stage_cols_cp(const Grp& G, float* S, int RGP, int R32, const float* M, int64_t ld,
+                                              int64_t col0, int ncol, const NodeRows& nr, int RG, bool vec) {
+    const int warp = G.tid >> 5, lane = G.tid & 31;
+    if (vec) {
+#pragma unroll
+        for (int a = 0; a < 4; ++a) {
+            const int jj = warp + 8 * a;
+            const float* mc = M + (col0 + min(jj, max(ncol - 1, 0))) * ld;
+#pragma unroll
+            for (int b = 0; b < 2; ++b) {
+                const int r = 4 * (lane + 32 * b);
+                if (r < R32) {
+                    const int valid = jj < ncol ? max(0, min(4, RG - r)) : 0;
+                    const float* src = valid > 0 ? mc + gathered_row(nr, r) : mc;
+                    const unsigned dst = (unsigned)__cvta_generic_to_shared(S + (size_t)jj * RGP + r);
+                    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src),
+                                 "r"(valid * 4)
+                                 : "memory");
+                }
+            }
+        }
+    } else {
+#pragma unroll
+        for (int a = 0; a < 4; ++a) {
+            const int jj = warp + 8 * a;
+            const float* mc = M + (col0 + min(jj, max(ncol - 1, 0))) * ld;
+#pragma unroll
+            for (int b = 0; b < 8; ++b) {
+                const int r = lane + 32 * b;
+                if (r < R32) {
+                    const bool valid = jj < ncol && r < RG;
+                    const float* src = valid ? mc + gathered_row(nr, r) : mc;
+                    const unsigned dst = (unsigned)__cvta_generic_to_shared(S + (size_t)jj * RGP + r);
+                    asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;" ::"r"(dst), "l"(src),
+                                 "r"(valid ? 4 : 0)
+                                 : "memory");
+                }
+            }
+        }
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
 }
 
 template <typename T>
@@ -919,6 +987,10 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
     T* Tt = Wp + 4 * 32 * kTS;
     T* W = Tt + 32 * kTS;
     T* tau_s = W + 32 * kTS;
+    // 16-byte staging / write-back of C blocks (fp32): A 16-byte aligned and
+    // every row segment (tiles, R slots) starting on a multiple of 4 rows
+    const bool vec = sizeof(T) == 4 && (reinterpret_cast<uintptr_t>(A) % 16 == 0) && (g.lda % 4 == 0) &&
+                     (g.row0 % 4 == 0) && (g.b % 4 == 0) && (g.bm % 4 == 0);
     __shared__ int s_task;
     const Grp G0{(int)threadIdx.x, 0};
     int* ticket = sync;
@@ -1048,7 +1120,13 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
             for (int ib = 0; ib < nblk; ++ib) {
                 const int64_t cb0 = tfirst + 32 * ((ib + 1) % nblk);
                 const int ncb = (int)(tend - cb0 < 32 ? tend - cb0 : 32);
-                stage_cols(G0, Cs, RGP, R32, static_cast<const T*>(A), g.lda, cb0, ncb, nr, RG, false, p);
+                const bool vec_p = vec && (nr.n0 % 4 == 0);
+                if constexpr (sizeof(T) == 4) {
+                    stage_cols_cp(G0, Cs, RGP, R32, A, g.lda, cb0, ncb, nr, RG, vec_p);
+                    asm volatile("cp.async.wait_group 0;" ::: "memory");
+                } else {
+                    stage_cols(G0, Cs, RGP, R32, static_cast<const T*>(A), g.lda, cb0, ncb, nr, RG, false, p);
+                }
                 __syncthreads();
                 CAQR_PROF(6);
                 if constexpr (sizeof(T) == 4)
@@ -1056,7 +1134,7 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
                 else
                     gemm_vtc(G0, P, Cs, RGP, R32, Wp, W);
                 CAQR_PROF(7);
-                apply_block(G0, P, Cs, Tt, W, RGP, R32, RG, wp, 1, nr, A, g.lda, cb0, ncb);
+                apply_block(G0, P, Cs, Tt, W, RGP, R32, RG, wp, 1, nr, A, g.lda, cb0, ncb, vec_p);
                 CAQR_PROF(8);
             }
             // ---- publish ----------------------------------------------------------
