@@ -61,6 +61,12 @@ constexpr int64_t kMaxLeaf = 256;     // tallest tile the kernels stage in share
 constexpr int64_t kFusedLeaf = 224;   // default tile height: [32 R rows; tile] fits 256 rows
 constexpr int64_t kChainTarget = 296; // chains per group (2 per B200 SM; device-independent constant)
 constexpr int64_t kStreamChains = 1184;  // skinny chains: 8 warps x 148 B200 SMs
+// CAQR_STREAM16=1: n <= 8 panels on 128-row tiles with 16 warps per SM
+// (2368 chains) instead of 256-row tiles with 8 warps per SM.
+static inline bool stream16_policy() {
+    const char* e = getenv("CAQR_STREAM16");
+    return e && e[0] == '1';
+}
 
 struct Plan {
     int64_t m = 0, n = 0;
@@ -89,9 +95,10 @@ static int make_plan(int64_t m, int64_t n, int dtype, const caqr_opts* o, int op
     // fewer, larger tasks win, e.g. 4096 x 16: 0.13 ms vs 0.26 ms measured)
     pl->skinny = dtype == CAQR_F32 && n <= 16 && nb >= n && m >= (int64_t(1) << 18);
     // streaming kernel: one chain per warp, 8 warps per SM (148 SMs)
-    pl->chain_target = pl->skinny ? kStreamChains : kChainTarget;
+    const bool s16 = pl->skinny && n <= 8 && stream16_policy();
+    pl->chain_target = pl->skinny ? (s16 ? 2 * kStreamChains : kStreamChains) : kChainTarget;
     int64_t b = (o && o->leaf_rows > 0) ? o->leaf_rows
-                                        : (pl->skinny ? (n <= 8 ? 256 : 128)
+                                        : (pl->skinny ? (n <= 8 && !s16 ? 256 : 128)
                                                       : (nb <= kFusedLeaf ? kFusedLeaf : kMaxLeaf));
     if (b % 32 != 0 || b > kMaxLeaf) return -opt_pos;
     b = std::max(b, round_up(nb, 32));
@@ -134,7 +141,15 @@ static inline size_t group_t_bytes(const Geom& G, size_t es) {
     return (size_t)2 * G.L * G.npan * kPW * kPW * es;
 }
 static inline size_t group_sync_bytes(const Geom& G) {
-    return (size_t)round_up((32 + G.L * G.npan) * (int64_t)sizeof(int), 256);
+    int64_t ints = 32 + G.L * G.npan;
+    // skinny groups: room for the streaming kernel's cross-CTA exchange area
+    // (one n x n R per CTA at sync + 64) and arrival counters (tsqr_stream.cuh)
+    if (G.npan == 1 && G.ncols <= 16) {
+        const int64_t nct = ceil_div(G.P, 8);  // CTAs of 8 (or 16) warps
+        const int64_t rx = G.ncols <= 8 ? stream_rx_ints<float, 8>(nct) : stream_rx_ints<float, 16>(nct);
+        ints = std::max<int64_t>(ints, 64 + rx + 16 * nct);
+    }
+    return (size_t)round_up(ints * (int64_t)sizeof(int), 256);
 }
 static inline size_t group_ws_bytes(const Geom& G, size_t es) {
     return group_t_bytes(G, es) + group_sync_bytes(G);
@@ -492,10 +507,15 @@ static int launch_stream(const Geom& G, T* A, T* Tws, int* sync, cudaStream_t s,
     if constexpr (sizeof(T) == 4) {
         const bool nc8 = G.ncols <= 8 && G.b == 256, nc16 = G.ncols <= 16 && G.b == 128;
         if (!nc8 && !nc16) return 0;
-        // the CTAs' packed R's travel through the workspace's flag area
-        const int64_t nct = ceil_div(G.P, 8), nc = nc8 ? 8 : 16;
-        if ((int64_t)sizeof(T) * nct * nc * (nc + 1) / 2 > (int64_t)sizeof(int) * (G.L * G.npan - 32)) return 0;
-        if ((nc8 ? stream_smem_bytes<T, 8, 8, 8>(nct) : stream_smem_bytes<T, 16, 4, 8>(nct)) > 220 * 1024) return 0;
+        const bool w16 = G.ncols <= 8 && G.b == 128;  // 16 warps x 128-row tiles (CAQR_STREAM16)
+        // the CTAs' R's travel through the workspace's flag area
+        const int64_t nct = ceil_div(G.P, w16 ? 16 : 8);
+        // (plus one arrival counter per (cross-CTA level, CTA))
+        const int64_t rx = (nc8 || w16) ? stream_rx_ints<T, 8>(nct) : stream_rx_ints<T, 16>(nct);
+        if ((64 + rx + (int64_t)tree_levels(G.P) * nct) * (int64_t)sizeof(int) > (int64_t)group_sync_bytes(G)) return 0;
+        if ((nc8 ? stream_smem_bytes<T, 8, 8, 8>(nct)
+                 : w16 ? stream_smem_bytes<T, 8, 4, 16>(nct) : stream_smem_bytes<T, 16, 4, 8>(nct)) > 220 * 1024)
+            return 0;
         // 16-byte cp.async needs every tile column start 16-byte aligned
         const bool vec = (reinterpret_cast<uintptr_t>(A) % 16 == 0) && (G.lda % 4 == 0) && (G.row0 % 4 == 0);
         cudaError_t e = cudaMemsetAsync(sync, 0, group_sync_bytes(G), s);
@@ -507,8 +527,9 @@ static int launch_stream(const Geom& G, T* A, T* Tws, int* sync, cudaStream_t s,
                 by = 2.0 * mr * nc * sizeof(T);
             }
             TraceScope ts(K_TSQR_SKINNY, fl, by, s);
-            e = nc8 ? launch_stream_nc<T, 8, 8>(G, A, Tws, sync, vec, s)
-                    : launch_stream_nc<T, 16, 4>(G, A, Tws, sync, vec, s);
+            e = nc8   ? launch_stream_nc<T, 8, 8>(G, A, Tws, sync, vec, s)
+                : w16 ? launch_stream_nc<T, 8, 4, 16>(G, A, Tws, sync, vec, s)
+                      : launch_stream_nc<T, 16, 4>(G, A, Tws, sync, vec, s);
         }
         if (e != cudaSuccess) {
             g_last_cuda_error = (int)e;

@@ -1,6 +1,7 @@
 // tsqr_stream.cuh -- streaming TSQR of a skinny panel (n <= 16): one WARP per
 // chain, the chain's R resident in shared memory, tiles double-buffered by
-// cp.async, the binary tree climbed by the last-arriving warp.
+// cp.async, each merge of the binary tree done by the second of its two
+// children to arrive (warps inside a CTA, then CTAs).
 //
 // For the s-step Krylov shape ("millions of rows by less than ten
 // columns") the factorization is a stream of A through HBM: read each tile
@@ -16,10 +17,9 @@
 //   * per reflector ONE n-value warp all-reduce gives the squared norm, the dot
 //     products with the later columns (matvec of P:L704-711 on the unscaled
 //     column) and the Gram entries of the compact-WY T;
-//   * then the chain's R goes to its slot and the warp walks up the binary
-//     tree: at each merge an arrival counter picks the SECOND warp to arrive,
-//     which merges the two n x n triangles ("factor_tree") at once
-//     -- no warp ever spins on a flag.
+//   * then the chains' R's are merged up the binary tree ("factor_tree",
+//     P:L658-663): inside the CTA level by level, across CTAs by whichever
+//     CTA arrives SECOND at a pair (arrival counter) -- no one spins on a flag.
 #pragma once
 #include "tsqr_fused.cuh"
 
@@ -83,6 +83,7 @@ struct alignas(16) StreamWarp {
     T buf[2][NC][B];   // double-buffered tile (column-major, B rows)
     T R[NC][NC + 1];   // chain / subtree R, R[j][k] (upper)
     T G[NC][NC + 1];   // Gram entries G[a][j] = v_a^T v_j (a < j)
+    T Rs[NC][NC + 1];  // a sibling CTA's R (cross-CTA merges)
     T tau[NC];
     T red[32];         // all-reduce scratch
     T bc[2 * NC + 4];  // merge broadcast: v_j, tau, ...
@@ -297,14 +298,39 @@ __device__ __forceinline__ void merge_group(bool on, int k, const T* Ra, const T
     __syncwarp();
 }
 
-// Shared memory of the last CTA's tree phase: every CTA's R (slot c * NW),
-// then per merge unit (a group of NC lanes) its G / tau / broadcast scratch.
+// A merge recorded for write-out after the climb: V_2 (V[k][i], rows i <= k
+// of column k), the Gram entries and tau that give its T.
+constexpr int kStreamMaxRec = 12;  // >= merges one warp can do (4 in-CTA + 8 cross-CTA levels)
 template <typename T, int NC>
-struct TreeUnit {
-    T G[NC][NC + 1];
+struct StreamRec {
+    T V[NC][NC];
+    T G[NC][NC];
     T tau[NC];
-    T bc[NC + 4];
+    int64_t sb;
 };
+template <typename T>
+__device__ __forceinline__ void store_v4(T* p, T a, T b, T c, T d) {
+    if constexpr (sizeof(T) == 4) {
+        *reinterpret_cast<float4*>(p) = make_float4(a, b, c, d);
+    } else {
+        p[0] = a, p[1] = b, p[2] = c, p[3] = d;
+    }
+}
+template <typename T>
+__device__ __forceinline__ void load_v4_cg(const T* p, T (&v)[4]) {
+    if constexpr (sizeof(T) == 4) {
+        const float4 q = __ldcg(reinterpret_cast<const float4*>(p));
+        v[0] = q.x, v[1] = q.y, v[2] = q.z, v[3] = q.w;
+    } else {
+        for (int e = 0; e < 4; ++e) v[e] = __ldcg(p + e);
+    }
+}
+
+// Ints of the workspace exchange area holding every CTA's R (NC x NC, 32-aligned).
+template <typename T, int NC>
+__host__ __device__ inline int64_t stream_rx_ints(int64_t nct) {
+    return ((nct * (NC * NC) * (int64_t)sizeof(T) / 4) + 31) & ~int64_t(31);
+}
 
 template <typename T, int NC, int RPL, int NW, bool VEC>
 __global__ void __launch_bounds__(32 * NW, 1)
@@ -315,7 +341,6 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
     constexpr int LDR = NC + 1;
     using SW = StreamWarp<T, NC, B>;
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    __shared__ int s_last;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     SW* Ws = reinterpret_cast<SW*>(smem_raw);
     SW& W = Ws[warp];
@@ -404,18 +429,44 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
         }
     }
 
-    // ---- tree levels inside the CTA: warps' R's in shared memory ----------
+    // ---- the binary tree over the chain R's -------------------
+    // A merge's V_2 and T are not needed by the levels above it (only its new
+    // R is), so they are recorded in the merging warp's free tile buffers and
+    // written out after the climb, by all warps of the CTA together.
+    // (NC <= 8; wider panels store at once: their records would not fit)
+    using Rec = StreamRec<T, NC>;
+    constexpr bool DEFER = NC <= 8;
+    static_assert(!DEFER || sizeof(Rec) * kStreamMaxRec <= sizeof(T) * 2 * NC * B, "records fit in the tile buffers");
+    __shared__ int s_nrec[NW];
+    int nrec = 0;
+    auto merge_rec = [&](const T* Ra, const T* Rb, int nb, T* Ro, int64_t sb) {
+        T rb[NC];
+        merge_group<T, NC>(lane < NC, lane, Ra, Rb, LDR, nb, Ro, rb, &W.G[0][0], LDR, W.tau, W.bc);
+        if (!DEFER || nrec >= kStreamMaxRec) {
+            store_merge(lane < NC, lane, sb, rb, &W.G[0][0], W.tau);
+            return;
+        }
+        Rec& r = reinterpret_cast<Rec*>(&W.buf[0][0][0])[nrec++];
+        if (lane < NC) {
+#pragma unroll
+            for (int i = 0; i < NC; ++i) {
+                r.V[lane][i] = rb[i];
+                r.G[i][lane] = W.G[i][lane];
+            }
+            r.tau[lane] = W.tau[lane];
+        }
+        if (lane == 0) r.sb = sb;
+        __syncwarp();
+    };
+    // inside the CTA: warps' R's in shared memory, level by level
     int l = 0;
     for (; (2 << l) <= NW && l < nlevels; ++l) {
         __syncthreads();
         const int hl = 1 << l;
         const bool on = __shfl_sync(0xffffffffu, (live && (warp & (2 * hl - 1)) == 0 && chain + hl < g.P) ? 1 : 0, 0);
         if (on) {  // warp-uniform
-            T rb[NC];
             const int64_t sb = chain + hl;
-            merge_group<T, NC>(lane < NC, lane, &W.R[0][0], &Ws[warp + hl].R[0][0], LDR,
-                               (int)min64(NC, slot_h(sb)), &W.R[0][0], rb, &W.G[0][0], LDR, W.tau, W.bc);
-            store_merge(lane < NC, lane, sb, rb, &W.G[0][0], W.tau);
+            merge_rec(&W.R[0][0], &Ws[warp + hl].R[0][0], (int)min64(NC, slot_h(sb)), &W.R[0][0], sb);
         }
     }
     __syncthreads();
@@ -430,127 +481,90 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
     };
     if (l >= nlevels) {  // the whole tree fitted in this CTA
         if (warp == 0) store_r(&W.R[0][0], base);
-        return;
-    }
-    // the CTA's R (packed upper triangle, contiguous per CTA) into the
-    // workspace's exchange area -- one coalesced read for the last CTA
-    constexpr int NP = NC * (NC + 1) / 2;
-    T* Rx = reinterpret_cast<T*>(sync + 64);
-    if (warp == 0 && lane < NC)
-#pragma unroll
-        for (int i = 0; i < NC; ++i)
-            if (i <= lane) Rx[blockIdx.x * NP + lane * (lane + 1) / 2 + i] = W.R[i][lane];
-
-    // ---- the last CTA to get here climbs the rest of the tree ---------------
-    __threadfence();
-    __syncthreads();
-    if (threadIdx.x == 0) s_last = atomicAdd(sync + 32, 1) == (int)gridDim.x - 1;
-    __syncthreads();
-    if (!s_last) return;
-    __threadfence();
-    const unsigned long long tt0 = prof ? gtime() : 0ull;
-    const int nct = (int)gridDim.x;
-    T* Rall = reinterpret_cast<T*>(smem_raw);  // [nct][NC][LDR]
-    using TU = TreeUnit<T, NC>;
-    TU* units = reinterpret_cast<TU*>(Rall + (size_t)nct * NC * LDR);
-    // merges whose V_2 / T stay in shared memory until the tree is done
-    // (NC <= 8): the tree's few global stores then leave in one burst instead
-    // of one round trip per level behind the chains' write-back
-    constexpr bool DEFER = NC <= 8;
-    T* Vd = reinterpret_cast<T*>(units + NW * (32 / NC));  // [nct][NP]
-    T* Td = Vd + (size_t)nct * NP;                         // [nct][NC][NC]
-    {   // every CTA's R: independent coalesced loads in batches, then the stores
-        constexpr int BATCH = 8;
-        const int total = nct * NP;
-        for (int e0 = threadIdx.x; e0 < total; e0 += 32 * NW * BATCH) {
-            T v[BATCH];
-#pragma unroll
-            for (int u = 0; u < BATCH; ++u) {
-                const int e = e0 + u * 32 * NW;
-                v[u] = e < total ? __ldcg(Rx + e) : T(0);
+    } else if (warp == 0) {
+        // ---- across CTAs: the SECOND CTA to finish a pair merges it --------
+        // Same pairs, order and storage as a level-by-level tree, but no CTA
+        // waits: each publishes its R in the workspace exchange area and takes
+        // a ticket on the pair's arrival counter; the first arriver stops, the
+        // second merges [R_a; R_b] and climbs on.  Only lanes that write the
+        // R fence, so the publish does not wait for earlier V/T stores.
+        const int nct = (int)gridDim.x;
+        constexpr int NQ = NC * NC / 4;  // float4's per R
+        T* Rx = reinterpret_cast<T*>(sync + 64);          // [nct][NC][NC]
+        int* cnt = sync + 64 + stream_rx_ints<T, NC>(nct);  // [levels][nct]
+        const int l0 = l;
+        int64_t cur = blockIdx.x;  // CTA whose slot (cur * NW) this R belongs to
+        T* Rm = &W.R[0][0];
+        T* Rs = &W.Rs[0][0];
+        bool root = true;
+        for (; l < nlevels; ++l) {
+            const int64_t hl = int64_t(1) << l;
+            const int64_t slot = cur * NW;
+            const bool left = ((slot >> l) & 1) == 0;
+            const int64_t sa = left ? slot : slot - hl, sb = sa + hl;
+            if (sb >= g.P) continue;  // no right member at this level: pass up
+            for (int q = lane; q < NQ; q += 32) {
+                const int i = (4 * q) / NC, c = (4 * q) % NC;
+                const T* rr = Rm + i * LDR + c;
+                store_v4<T>(Rx + cur * NC * NC + 4 * q, rr[0], rr[1], rr[2], rr[3]);
+                __threadfence();
             }
-#pragma unroll
-            for (int u = 0; u < BATCH; ++u) {
-                const int e = e0 + u * 32 * NW;
-                if (e < total) {
-                    const int c = e / NP, q = e % NP;
-                    int kk = 0;
-                    while ((kk + 1) * (kk + 2) / 2 <= q) ++kk;
-                    const int i = q - kk * (kk + 1) / 2;
-                    Rall[(size_t)c * NC * LDR + i * LDR + kk] = v[u];
-                }
+            __syncwarp();
+            int old = 0;
+            if (lane == 0) old = atomicAdd(cnt + (int64_t)(l - l0) * nct + sa / NW, 1);
+            old = __shfl_sync(0xffffffffu, old, 0);
+            if (old == 0) {  // the sibling merges
+                root = false;
+                break;
             }
+            __threadfence();
+            const int64_t other = (left ? sb : sa) / NW;
+            for (int q = lane; q < NQ; q += 32) {
+                const int i = (4 * q) / NC, c = (4 * q) % NC;
+                T v[4];
+                load_v4_cg<T>(Rx + other * NC * NC + 4 * q, v);
+#pragma unroll
+                for (int e = 0; e < 4; ++e) Rs[i * LDR + c + e] = v[e];
+            }
+            __syncwarp();
+            merge_rec(left ? Rm : Rs, left ? Rs : Rm, (int)min64(NC, slot_h(sb)), Rm, sb);
+            cur = sa / NW;
         }
-        for (int e = threadIdx.x; e < nct * NC * NC; e += 32 * NW) {  // strict lower parts
-            const int c = e / (NC * NC), i = (e / NC) % NC, kk = e % NC;
-            if (i > kk) Rall[(size_t)c * NC * LDR + i * LDR + kk] = T(0);
+        if (root) {
+            store_r(Rm, 0);  // the root R into A's top rows
+            if (prof && lane == 0) atomicMax(prof + 2, gtime());
         }
     }
-    if (prof && threadIdx.x == 0) prof[7] = gtime() - tt0;
-    const long long cl0 = clock64();
-    constexpr int GPW = 32 / NC;  // merge groups per warp
-    const int grp = lane / NC, k = lane % NC;
-    const int unit = warp * GPW + grp;
-    TU& U = units[unit];
-    for (; l < nlevels; ++l) {
-        __syncthreads();
-        const int64_t hl = int64_t(1) << l;
-        const int64_t nm = (g.P - 1 >= hl) ? (g.P - 1 - hl) / (2 * hl) + 1 : 0;
-        for (int64_t r0 = 0; r0 < nm; r0 += NW * GPW) {  // rounds of NW*GPW merges (warp-uniform loop)
-            const int64_t node = r0 + unit;
-            const bool on = node < nm;
-            const int64_t sa = node << (l + 1), sb = sa + hl;
-            const int ca = on ? (int)(sa / NW) : 0, cb = on ? (int)(sb / NW) : 0;
-            T rb[NC];
-            T* Ra = Rall + (size_t)ca * NC * LDR;
-            const long long c0 = clock64();
-            if (!(dbg & 2))
-            merge_group<T, NC>(on, k, Ra, Rall + (size_t)cb * NC * LDR, LDR,
-                               on ? (int)min64(NC, slot_h(sb)) : 0, Ra, rb, &U.G[0][0], LDR, U.tau, U.bc);
-            const long long c1 = clock64();
-            if (prof && threadIdx.x == 0) { prof[9] += c1 - c0; prof[12] += 1; }
-            if (dbg & 1) {
-            } else if (DEFER) {
-                if (on)
+    // ---- write out every recorded merge (V_2 into R_b's slot, T), CTA-wide
+    if (lane == 0) s_nrec[warp] = nrec;
+    __syncthreads();
+    {
+        int idx = 0;
+        for (int w = 0; w < NW; ++w) {
+            const int nw = s_nrec[w];
+            const Rec* rs = reinterpret_cast<const Rec*>(&Ws[w].buf[0][0][0]);
+            for (int r = 0; r < nw; ++r, ++idx) {
+                if (idx % NW != warp) continue;
+                const Rec& rc = rs[r];
+                const int64_t sb = rc.sb;
+                const int k = lane;
+                const int64_t hb = slot_h(sb);
+                if (k < NC && k < wp) {
+                    T* bb = slot_ptr(sb) + k * g.lda;
 #pragma unroll
                     for (int i = 0; i < NC; ++i)
-                        if (i <= k) Vd[(size_t)cb * NP + k * (k + 1) / 2 + i] = rb[i];
-                stream_write_t<T, NC>(on, k, &U.G[0][0], LDR, U.tau, wp, Td + (size_t)cb * NC * NC, NC);
-                __syncwarp();
-                if (prof && threadIdx.x == 0) prof[10] += clock64() - c1;
-            } else {
-                store_merge(on, k, sb, rb, &U.G[0][0], U.tau);
+                        if (i <= k && i < hb) bb[i] = rc.V[k][i];
+                }
+                stream_write_t<T, NC>(k < NC, k, &rc.G[0][0], NC, rc.tau, wp,
+                                      Tws + ((g.L + sb * g.K) * g.npan) * (kPW * kPW));
             }
-            if (prof && on && k == 0) atomicAdd(prof + 6, 1ull);
         }
-    }
-    __syncthreads();
-    if (prof && threadIdx.x == 0) prof[11] = clock64() - cl0;
-    if (warp == 0) store_r(Rall, 0);  // the root R
-    if (DEFER && !(dbg & 1)) {  // V_2 into every R_b slot (CTA c >= 1), T blocks
-        for (int e = threadIdx.x; e < nct * NC * NC; e += 32 * NW) {
-            const int c = e / (NC * NC), j = (e / NC) % NC, kk = e % NC;  // T[kk][j] / V_2 (j, kk)
-            if (c == 0) continue;
-            const int64_t sb = (int64_t)c * NW;
-            if (j < wp && kk < wp)
-                Tws[((g.L + sb * g.K) * g.npan) * (kPW * kPW) + j * kPW + kk] = Td[(size_t)c * NC * NC + j * NC + kk];
-            if (j <= kk && kk < wp && j < slot_h(sb))
-                slot_ptr(sb)[kk * g.lda + j] = Vd[(size_t)c * NP + kk * (kk + 1) / 2 + j];
-        }
-    }
-    if (prof && threadIdx.x == 0) {
-        const unsigned long long te = gtime();
-        atomicAdd(prof + 5, te - tt0);
-        atomicMax(prof + 2, te);
     }
 }
 
 template <typename T, int NC, int RPL, int NW>
-inline size_t stream_smem_bytes(int64_t nct) {
-    const size_t chain = sizeof(StreamWarp<T, NC, 32 * RPL>) * NW;
-    const size_t tree = sizeof(T) * (size_t)nct * NC * (NC + 1) + sizeof(TreeUnit<T, NC>) * NW * (32 / NC) +
-                        (NC <= 8 ? sizeof(T) * (size_t)nct * (NC * (NC + 1) / 2 + NC * NC) : 0);
-    return chain > tree ? chain : tree;
+inline size_t stream_smem_bytes(int64_t /*nct*/) {
+    return sizeof(StreamWarp<T, NC, 32 * RPL>) * NW;
 }
 
 }  // namespace caqr
