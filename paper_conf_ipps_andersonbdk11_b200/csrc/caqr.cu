@@ -144,7 +144,7 @@ static inline size_t group_sync_bytes(const Geom& G) {
     int64_t ints = 32 + G.L * G.npan;
     // skinny groups: room for the streaming kernel's cross-CTA exchange area
     // (one n x n R per CTA at sync + 64) and arrival counters (tsqr_stream.cuh)
-    if (G.npan == 1 && G.ncols <= 16) {
+    if (G.npan == 1 && ((G.ncols <= 8 && (G.b == 256 || G.b == 128)) || (G.ncols <= 16 && G.b == 128))) {
         const int64_t nct = ceil_div(G.P, 8);  // CTAs of 8 (or 16) warps
         const int64_t rx = G.ncols <= 8 ? stream_rx_ints<float, 8>(nct) : stream_rx_ints<float, 16>(nct);
         ints = std::max<int64_t>(ints, 64 + rx + 16 * nct);
