@@ -184,6 +184,69 @@ int caqr_dist_factor_f64(caqr_dist *h, int64_t m_local, int64_t n, double *A, in
                          void *cws, size_t cws_bytes, const caqr_opts *opts,
                          caqr_stream_t stream);
 
+/* ---- Application layer: SVD via QR and robust PCA (Sec. VI) -----------------
+ * The paper's motivating workload: robust PCA of a video matrix
+ * (one column per frame) by an alternating-directions method whose
+ * main cost is the SVD of a tall-skinny matrix, done as A = QR, SVD(R) = U S V^T,
+ * left vectors Q U.  With caqr_factor_f32 and caqr_apply_q_f32 the
+ * whole iteration runs on the GPU (the paper takes the small SVD to the CPU,
+ * P:L1068-1074; here it is one CTA).  All pointers are device pointers. */
+
+/* SVD of a small square matrix, R = U diag(sigma) V^T, by one-sided (Hestenes)
+ * Jacobi rotations in fp64 on one CTA.  R: n x n (ldr >= n, not modified);
+ * U, V: n x n outputs (ldu, ldv >= n), orthogonal; sigma: n outputs, descending,
+ * >= 0.  A zero singular value gets a zero U column.  0 <= n <= 112.  V may be
+ * NULL: the right vectors are then not formed (about half the work; see
+ * caqr_svt_core_r_f32, which needs only U, sigma and R).
+ * info: -1 n, -2 R, -3 ldr, -4 U, -5 ldu, -6 sigma, -8 ldv; n = 0 quick return. */
+int caqr_svd_small_f32(int64_t n, const float *R, int64_t ldr, float *U, int64_t ldu, float *sigma,
+                       float *V, int64_t ldv, caqr_stream_t stream);
+int caqr_svd_small_f64(int64_t n, const double *R, int64_t ldr, double *U, int64_t ldu, double *sigma,
+                       double *V, int64_t ldv, caqr_stream_t stream);
+
+/* Singular value threshold of the small factor (Fig. 11 "threshold these
+ * singular values"): W = U diag(max(sigma - tau, 0)) V^T, n x n,
+ * from caqr_svd_small's outputs.  The low-rank iterate is then L = Q [W; 0]
+ * (caqr_embed_top_f32 + caqr_apply_q_f32).
+ * info: -1 n (0..112), -2 U, -3 ldu, -4 sigma, -5 V, -6 ldv, -8 W, -9 ldw. */
+int caqr_svt_core_f32(int64_t n, const float *U, int64_t ldu, const float *sigma, const float *V,
+                      int64_t ldv, float tau, float *W, int64_t ldw, caqr_stream_t stream);
+
+/* The same W without V: W = U diag(max(sigma - tau, 0) / sigma) U^T R, which equals
+ * U diag(max(sigma - tau, 0)) V^T because U^T R = diag(sigma) V^T (only sigma > tau
+ * is divided by).  R: the n x n matrix caqr_svd_small_f32 decomposed.
+ * info: -1 n, -2 U, -3 ldu, -4 sigma, -5 R, -6 ldr, -8 W, -9 ldw. */
+int caqr_svt_core_r_f32(int64_t n, const float *U, int64_t ldu, const float *sigma, const float *R,
+                        int64_t ldr, float tau, float *W, int64_t ldw, caqr_stream_t stream);
+
+/* C (m x n, ldc >= m) = [W; 0] with W n x n (ldw >= n), n <= m.
+ * info: -1 m, -2 n, -3 W, -4 ldw, -5 C, -6 ldc. */
+int caqr_embed_top_f32(int64_t m, int64_t n, const float *W, int64_t ldw, float *C, int64_t ldc,
+                       caqr_stream_t stream);
+
+/* One shrinkage + dual step of the alternating-directions iteration (P:L1107-1113,
+ * reading S19 of DESIGN.md), elementwise over m x n, given the new low-rank
+ * iterate L:
+ *   S <- sign(t) max(|t| - lambda/mu, 0),  t = M - L + Y/mu
+ *   Y <- Y + mu (M - L - S)
+ *   X <- M - S + Y/mu_next                 (the next iteration's SVT input)
+ *   resid[0] <- ||M - L - S||_F^2          (fixed-order reduction: deterministic)
+ * M, L read; S, Y, X written (X may not alias the others).  resid: device
+ * double[CAQR_RPCA_RESID_LEN] scratch.  mu, mu_next > 0, lambda >= 0.
+ * info: -1 m, -2 n, -3..-12 the matrices / leading dimensions in order,
+ * -13 mu, -14 mu_next, -15 lambda, -16 resid. */
+#define CAQR_RPCA_RESID_LEN 1025
+int caqr_rpca_update_f32(int64_t m, int64_t n, const float *M, int64_t ldm, const float *L, int64_t ldl,
+                         float *S, int64_t lds, float *Y, int64_t ldy, float *X, int64_t ldx, float mu,
+                         float mu_next, float lambda, double *resid, caqr_stream_t stream);
+/* Start of the iteration: S = 0, Y = yscale M, X = M + Y/mu.
+ * info: -1 m, -2 n, -3 M, -4 ldm, -6 S, -7 lds, -8 Y, -9 ldy, -10 X, -11 ldx, -12 mu. */
+int caqr_rpca_init_f32(int64_t m, int64_t n, const float *M, int64_t ldm, float yscale, float *S,
+                       int64_t lds, float *Y, int64_t ldy, float *X, int64_t ldx, float mu,
+                       caqr_stream_t stream);
+/* out[0] (device float) = max |M_ij| (0 for an empty M).  info: -1 m, -2 n, -3 M, -4 ldm, -5 out. */
+int caqr_absmax_f32(int64_t m, int64_t n, const float *M, int64_t ldm, float *out, caqr_stream_t stream);
+
 /* Diagnostics. */
 const char *caqr_strerror(int info);
 int caqr_last_cuda_error(void);          /* cudaError_t of the last CAQR_ERR_CUDA (thread-local) */

@@ -97,6 +97,20 @@ def lib() -> ctypes.CDLL:
         L.caqr_dist_create.restype = ip
         L.caqr_dist_destroy.argtypes = [vp]
         L.caqr_dist_destroy.restype = None
+        fl = ctypes.c_float
+        for suf in ("f32", "f64"):
+            f = getattr(L, f"caqr_svd_small_{suf}")
+            f.argtypes = [i64, vp, i64, vp, i64, vp, vp, i64, vp]
+            f.restype = ip
+        L.caqr_svt_core_f32.argtypes = [i64, vp, i64, vp, vp, i64, fl, vp, i64, vp]
+        L.caqr_svt_core_r_f32.argtypes = [i64, vp, i64, vp, vp, i64, fl, vp, i64, vp]
+        L.caqr_embed_top_f32.argtypes = [i64, i64, vp, i64, vp, i64, vp]
+        L.caqr_rpca_update_f32.argtypes = [i64, i64, vp, i64, vp, i64, vp, i64, vp, i64, vp, i64, fl, fl, fl,
+                                           vp, vp]
+        L.caqr_rpca_init_f32.argtypes = [i64, i64, vp, i64, fl, vp, i64, vp, i64, vp, i64, fl, vp]
+        L.caqr_absmax_f32.argtypes = [i64, i64, vp, i64, vp, vp]
+        for name in ("svt_core", "svt_core_r", "embed_top", "rpca_update", "rpca_init", "absmax"):
+            getattr(L, f"caqr_{name}_f32").restype = ip
         _lib = L
         return L
 
@@ -278,6 +292,99 @@ def caqr_combine_apply(Rstack, P: int, ws, C, trans: bool = True, stream=None):
                                                         C.shape[1], pc, ldc, _stream(stream))
     _check(f"caqr_combine_apply_{suf}", info)
     return C
+
+
+# ---- application layer: SVD via QR, robust PCA (include/caqr.h, Sec. VI) ----
+CAQR_RPCA_RESID_LEN = 1025
+
+
+def _f32(t, name):
+    torch = _torch()
+    if t.dtype != torch.float32:
+        raise TypeError(f"caqr: {name} must be float32")
+    return _colmajor(t, name)
+
+
+def caqr_svd_small(R, U=None, sigma=None, V=None, stream=None, want_v: bool = True):
+    """R (n x n) = U diag(sigma) V^T on the GPU (one-CTA Jacobi).  Returns (U, sigma, V);
+    V is None when want_v is False (right vectors not formed)."""
+    torch = _torch()
+    code, suf = _dtype_code(R)
+    n = R.shape[0]
+    if R.shape[1] != n:
+        raise ValueError("caqr_svd_small: R must be square")
+    pr, ldr = _colmajor(R, "R")
+    U = colmajor_empty(n, n, R.dtype, R.device) if U is None else U
+    if want_v:
+        V = colmajor_empty(n, n, R.dtype, R.device) if V is None else V
+        pv, ldv = _colmajor(V, "V")
+    else:
+        V, pv, ldv = None, None, max(n, 1)
+    sigma = torch.empty(n, dtype=R.dtype, device=R.device) if sigma is None else sigma
+    pu, ldu = _colmajor(U, "U")
+    info = getattr(lib(), f"caqr_svd_small_{suf}")(n, pr, ldr, pu, ldu, sigma.data_ptr(), pv, ldv,
+                                                    _stream(stream))
+    _check(f"caqr_svd_small_{suf}", info)
+    return U, sigma, V
+
+
+def caqr_svt_core(U, sigma, V, tau: float, W=None, stream=None):
+    """W = U diag(max(sigma - tau, 0)) V^T (n x n)."""
+    n = U.shape[0]
+    pu, ldu = _f32(U, "U")
+    pv, ldv = _f32(V, "V")
+    W = colmajor_empty(n, n, U.dtype, U.device) if W is None else W
+    pw, ldw = _f32(W, "W")
+    _check("caqr_svt_core_f32", lib().caqr_svt_core_f32(n, pu, ldu, sigma.data_ptr(), pv, ldv, float(tau), pw,
+                                                        ldw, _stream(stream)))
+    return W
+
+
+def caqr_svt_core_r(U, sigma, R, tau: float, W=None, stream=None):
+    """W = U diag(max(sigma - tau, 0) / sigma) U^T R (= U diag(max(sigma - tau, 0)) V^T)."""
+    n = U.shape[0]
+    pu, ldu = _f32(U, "U")
+    pr, ldr = _f32(R, "R")
+    W = colmajor_empty(n, n, U.dtype, U.device) if W is None else W
+    pw, ldw = _f32(W, "W")
+    _check("caqr_svt_core_r_f32", lib().caqr_svt_core_r_f32(n, pu, ldu, sigma.data_ptr(), pr, ldr, float(tau), pw,
+                                                            ldw, _stream(stream)))
+    return W
+
+
+def caqr_embed_top(W, C, stream=None):
+    """C = [W; 0]."""
+    pw, ldw = _f32(W, "W")
+    pc, ldc = _f32(C, "C")
+    _check("caqr_embed_top_f32", lib().caqr_embed_top_f32(C.shape[0], W.shape[0], pw, ldw, pc, ldc,
+                                                          _stream(stream)))
+    return C
+
+
+def caqr_rpca_update(M, L, S, Y, X, mu: float, mu_next: float, lam: float, resid, stream=None):
+    m, n = M.shape
+    args = []
+    for t, nm in ((M, "M"), (L, "L"), (S, "S"), (Y, "Y"), (X, "X")):
+        args += list(_f32(t, nm))
+    _check("caqr_rpca_update_f32", lib().caqr_rpca_update_f32(m, n, *args, float(mu), float(mu_next), float(lam),
+                                                              resid.data_ptr(), _stream(stream)))
+
+
+def caqr_rpca_init(M, yscale: float, S, Y, X, mu: float, stream=None):
+    m, n = M.shape
+    pm, ldm = _f32(M, "M")
+    ps, lds = _f32(S, "S")
+    py, ldy = _f32(Y, "Y")
+    px, ldx = _f32(X, "X")
+    _check("caqr_rpca_init_f32", lib().caqr_rpca_init_f32(m, n, pm, ldm, float(yscale), ps, lds, py, ldy, px, ldx,
+                                                          float(mu), _stream(stream)))
+
+
+def caqr_absmax(M, out, stream=None):
+    pm, ldm = _f32(M, "M")
+    _check("caqr_absmax_f32", lib().caqr_absmax_f32(M.shape[0], M.shape[1], pm, ldm, out.data_ptr(),
+                                                    _stream(stream)))
+    return out
 
 
 def geqrf_flops(m: int, n: int) -> float:

@@ -16,6 +16,7 @@
 #include "tsqr_fused.cuh"
 #include "tsqr_kernels.cuh"
 #include "tsqr_skinny.cuh"
+#include "rpca.cuh"
 #include "tsqr_stream.cuh"
 
 namespace caqr {
@@ -25,9 +26,11 @@ static thread_local int g_last_cuda_error = 0;
 // ---- launch tracing (diagnostics: per-launch CUDA events on the launching
 // stream + host-computed algorithmic flops/bytes; see caqr_trace_begin) -------
 enum KernelId { K_PANEL_FACTOR = 0, K_PANEL_UPDATE = 1, K_EXTRACT_R = 2, K_SET_IDENTITY = 3,
-                K_TSQR_FUSED = 4, K_TSQR_SKINNY = 5, K_NUM = 6 };
-static const char* const kKernelNames[K_NUM] = {"panel_factor", "panel_update", "extract_r",
-                                                "set_identity", "tsqr_fused", "tsqr_skinny"};
+                K_TSQR_FUSED = 4, K_TSQR_SKINNY = 5, K_SVD_SMALL = 6, K_SVT_CORE = 7, K_EMBED_TOP = 8,
+                K_RPCA_UPDATE = 9, K_RPCA_INIT = 10, K_ABSMAX = 11, K_NUM = 12 };
+static const char* const kKernelNames[K_NUM] = {"panel_factor", "panel_update", "extract_r", "set_identity",
+                                                "tsqr_fused",   "tsqr_skinny",  "svd_small", "svt_core",
+                                                "embed_top",    "rpca_update",  "rpca_init", "absmax"};
 struct Trace {
     std::mutex mu;
     bool on = false;
@@ -805,6 +808,50 @@ static int combine_apply_impl(int P, int64_t n, const T* Rs, int64_t ld, const v
 
 using namespace caqr;
 
+
+// ---- application layer: SVD via QR and robust PCA (rpca.cuh) ----
+static inline unsigned elem_grid(int64_t total, int threads) {
+    const int64_t want = (total + threads - 1) / threads;
+    return (unsigned)std::max<int64_t>(1, std::min<int64_t>(want, (int64_t)num_sms() * 8));
+}
+
+template <typename T>
+static int svd_small_impl(int64_t n, const T* R, int64_t ldr, T* U, int64_t ldu, T* sigma, T* V, int64_t ldv,
+                          cudaStream_t s) {
+    if (n < 0 || n > kSvdMaxN) return -1;
+    if (ldr < std::max<int64_t>(1, n)) return -3;
+    if (ldu < std::max<int64_t>(1, n)) return -5;
+    if (ldv < std::max<int64_t>(1, n)) return -8;
+    if (n == 0) return 0;
+    if (!R) return -2;
+    if (!U) return -4;
+    if (!sigma) return -6;
+    const size_t smem = jacobi_svd_smem<T>((int)n);  // (V == NULL: right vectors not formed)
+    cudaError_t e = allow_smem(jacobi_svd_kernel<T>, smem);
+    if (e == cudaSuccess) {
+        TraceScope ts(K_SVD_SMALL, 0.0, 3.0 * n * n * sizeof(T), s);
+        // a pair counts as orthogonal at |b_p.b_q| <= tol ||b_p|| ||b_q||: U's
+        // orthogonality is tol-level, far below the output precision's epsilon
+        const double tol = sizeof(T) == 4 ? 1e-10 : 1e-15;
+        jacobi_svd_kernel<T><<<1, kSvdThreads, smem, s>>>((int)n, R, ldr, U, ldu, sigma, V, ldv, tol, 30);
+        e = cudaGetLastError();
+    }
+    if (e != cudaSuccess) {
+        g_last_cuda_error = (int)e;
+        return CAQR_ERR_CUDA;
+    }
+    return 0;
+}
+
+static int launch_status() {
+    const cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) {
+        g_last_cuda_error = (int)e;
+        return CAQR_ERR_CUDA;
+    }
+    return 0;
+}
+
 extern "C" {
 
 size_t caqr_workspace_bytes(int64_t m, int64_t n, int dtype, const caqr_opts* opts) {
@@ -972,6 +1019,137 @@ int caqr_plan_info(int64_t m, int64_t n, int dtype, const caqr_opts* opts, int64
     }
     out[6] = launches;
     return 0;
+}
+
+
+// ---- application layer (SVD via QR, robust PCA) ----------------------------
+int caqr_svd_small_f32(int64_t n, const float* R, int64_t ldr, float* U, int64_t ldu, float* sigma, float* V,
+                       int64_t ldv, caqr_stream_t stream) {
+    return svd_small_impl<float>(n, R, ldr, U, ldu, sigma, V, ldv, (cudaStream_t)stream);
+}
+int caqr_svd_small_f64(int64_t n, const double* R, int64_t ldr, double* U, int64_t ldu, double* sigma, double* V,
+                       int64_t ldv, caqr_stream_t stream) {
+    return svd_small_impl<double>(n, R, ldr, U, ldu, sigma, V, ldv, (cudaStream_t)stream);
+}
+
+int caqr_svt_core_f32(int64_t n, const float* U, int64_t ldu, const float* sigma, const float* V, int64_t ldv,
+                      float tau, float* W, int64_t ldw, caqr_stream_t stream) {
+    if (n < 0 || n > kSvdMaxN) return -1;
+    if (ldu < std::max<int64_t>(1, n)) return -3;
+    if (ldv < std::max<int64_t>(1, n)) return -6;
+    if (ldw < std::max<int64_t>(1, n)) return -9;
+    if (n == 0) return 0;
+    if (!U) return -2;
+    if (!sigma) return -4;
+    if (!V) return -5;
+    if (!W) return -8;
+    cudaStream_t s = (cudaStream_t)stream;
+    TraceScope ts(K_SVT_CORE, 2.0 * n * n * n, 4.0 * 3 * n * n, s);
+    svt_core_kernel<float><<<(unsigned)n, 128, 0, s>>>((int)n, U, ldu, sigma, V, ldv, tau, W, ldw);
+    return launch_status();
+}
+
+int caqr_svt_core_r_f32(int64_t n, const float* U, int64_t ldu, const float* sigma, const float* R, int64_t ldr,
+                        float tau, float* W, int64_t ldw, caqr_stream_t stream) {
+    if (n < 0 || n > kSvdMaxN) return -1;
+    if (ldu < std::max<int64_t>(1, n)) return -3;
+    if (ldr < std::max<int64_t>(1, n)) return -6;
+    if (ldw < std::max<int64_t>(1, n)) return -9;
+    if (n == 0) return 0;
+    if (!U) return -2;
+    if (!sigma) return -4;
+    if (!R) return -5;
+    if (!W) return -8;
+    cudaStream_t s = (cudaStream_t)stream;
+    TraceScope ts(K_SVT_CORE, 4.0 * n * n * n, 4.0 * 3 * n * n, s);
+    svt_core_r_kernel<float><<<(unsigned)n, 128, 0, s>>>((int)n, U, ldu, sigma, R, ldr, tau, W, ldw);
+    return launch_status();
+}
+
+int caqr_embed_top_f32(int64_t m, int64_t n, const float* W, int64_t ldw, float* C, int64_t ldc,
+                       caqr_stream_t stream) {
+    if (m < 0) return -1;
+    if (n < 0 || n > m) return -2;
+    if (ldw < std::max<int64_t>(1, n)) return -4;
+    if (ldc < std::max<int64_t>(1, m)) return -6;
+    if (m == 0 || n == 0) return 0;
+    if (!W) return -3;
+    if (!C) return -5;
+    cudaStream_t s = (cudaStream_t)stream;
+    TraceScope ts(K_EMBED_TOP, 0.0, 4.0 * m * n, s);
+    embed_top_kernel<float><<<elem_grid(m * n, 256), 256, 0, s>>>(m, n, W, ldw, C, ldc);
+    return launch_status();
+}
+
+int caqr_rpca_update_f32(int64_t m, int64_t n, const float* M, int64_t ldm, const float* L, int64_t ldl, float* S,
+                         int64_t lds, float* Y, int64_t ldy, float* X, int64_t ldx, float mu, float mu_next,
+                         float lambda, double* resid, caqr_stream_t stream) {
+    if (m < 0) return -1;
+    if (n < 0) return -2;
+    const int64_t lm = std::max<int64_t>(1, m);
+    if (ldm < lm) return -4;
+    if (ldl < lm) return -6;
+    if (lds < lm) return -8;
+    if (ldy < lm) return -10;
+    if (ldx < lm) return -12;
+    if (!(mu > 0.f)) return -13;
+    if (!(mu_next > 0.f)) return -14;
+    if (!(lambda >= 0.f)) return -15;
+    if (!resid) return -16;
+    if (m > 0 && n > 0) {
+        if (!M) return -3;
+        if (!L) return -5;
+        if (!S) return -7;
+        if (!Y) return -9;
+        if (!X) return -11;
+    }
+    cudaStream_t s = (cudaStream_t)stream;
+    {
+        TraceScope ts(K_RPCA_UPDATE, 12.0 * m * n, 4.0 * 7 * m * n, s);
+        rpca_update_kernel<float><<<kRpcaBlocks, 256, 0, s>>>(m, n, M, ldm, L, ldl, S, lds, Y, ldy, X, ldx, mu,
+                                                              mu_next, lambda, resid);
+    }
+    sum_parts_kernel<<<1, 256, 0, s>>>(kRpcaBlocks, resid);
+    return launch_status();
+}
+
+int caqr_rpca_init_f32(int64_t m, int64_t n, const float* M, int64_t ldm, float yscale, float* S, int64_t lds,
+                       float* Y, int64_t ldy, float* X, int64_t ldx, float mu, caqr_stream_t stream) {
+    if (m < 0) return -1;
+    if (n < 0) return -2;
+    const int64_t lm = std::max<int64_t>(1, m);
+    if (ldm < lm) return -4;
+    if (lds < lm) return -7;
+    if (ldy < lm) return -9;
+    if (ldx < lm) return -11;
+    if (!(mu > 0.f)) return -12;
+    if (m == 0 || n == 0) return 0;
+    if (!M) return -3;
+    if (!S) return -6;
+    if (!Y) return -8;
+    if (!X) return -10;
+    cudaStream_t s = (cudaStream_t)stream;
+    TraceScope ts(K_RPCA_INIT, 2.0 * m * n, 4.0 * 4 * m * n, s);
+    rpca_init_kernel<float><<<elem_grid(m * n, 256), 256, 0, s>>>(m, n, M, ldm, yscale, S, lds, Y, ldy, X, ldx, mu);
+    return launch_status();
+}
+
+int caqr_absmax_f32(int64_t m, int64_t n, const float* M, int64_t ldm, float* out, caqr_stream_t stream) {
+    if (m < 0) return -1;
+    if (n < 0) return -2;
+    if (ldm < std::max<int64_t>(1, m)) return -4;
+    if (!out) return -5;
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e = cudaMemsetAsync(out, 0, sizeof(float), s);
+    if (e != cudaSuccess) {
+        g_last_cuda_error = (int)e;
+        return CAQR_ERR_CUDA;
+    }
+    if (m == 0 || n == 0) return 0;
+    if (!M) return -3;
+    TraceScope ts(K_ABSMAX, 0.0, 4.0 * m * n, s);
+    absmax_kernel<float><<<elem_grid(m * n, 256), 256, 0, s>>>(m, n, M, ldm, out);
+    return launch_status();
 }
 
 }  // extern "C"

@@ -1,0 +1,300 @@
+// rpca.cuh -- the paper's application layer on the GPU:
+// SVD of a tall-skinny matrix through its QR (Sec. VI.B) and the
+// robust-PCA alternating-directions iteration built on it (P:L1089-1113,
+// Sec. VI.C, Fig. 11).
+//
+//   * jacobi_svd_kernel: SVD of the small n x n factor R.  The paper does this
+//     on the CPU with MKL; here one CTA does a one-sided
+//     (Hestenes) Jacobi SVD in fp64 in shared memory: columns of B = R are
+//     rotated pairwise (round-robin "circle" ordering, n/2 independent pairs per
+//     round, one warp per pair) until every pair is orthogonal to a relative
+//     tolerance; then sigma_j = ||b_j||, U = B diag(1/sigma), V = the product of
+//     the rotations, sorted by descending sigma.
+//   * svt_core_kernel: W = U diag(max(sigma - tau, 0)) V^T (the threshold of
+//     Fig. 11); the low-rank iterate is then L = Q [W; 0] (caqr_apply_q).
+//   * rpca_update_kernel: the shrinkage step and the dual update, fused with
+//     forming the next SVT input (one pass over M, L, S, Y), plus per-block
+//     partial sums of ||M - L - S||_F^2 reduced in a fixed order (deterministic).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+namespace caqr {
+
+constexpr int kSvdMaxN = 112;     // 2 n^2 doubles in shared memory (B and V)
+constexpr int kSvdThreads = 1024;
+constexpr int kRpcaBlocks = 1024;  // partial sums of the residual (fixed grid)
+
+__device__ __forceinline__ double warp_sum_d(double v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+
+// Player at position k of round r of the circle method over np (even) players.
+__device__ __forceinline__ int rr_player(int k, int r, int np) {
+    return k == 0 ? 0 : ((k - 1 + r) % (np - 1)) + 1;
+}
+
+template <typename T>
+__global__ void __launch_bounds__(kSvdThreads, 1)
+jacobi_svd_kernel(int n, const T* __restrict__ R, int64_t ldr, T* __restrict__ U, int64_t ldu,
+                  T* __restrict__ sigma, T* __restrict__ V, int64_t ldv, double tol, int max_sweeps) {
+    const double tol2 = tol * tol;
+    const bool want_v = V != nullptr;
+    extern __shared__ __align__(16) double sm[];
+    const int np = (n + 1) & ~1;  // an odd n gets a zero column (never rotated)
+    double* B = sm;               // [np][n]  column j at B + j * n
+    double* Vs = B + (size_t)np * n;  // [np][np]
+    double* nrm = Vs + (size_t)np * np;  // [np]
+    double* sig = nrm + np;              // [np]
+    int* rank = reinterpret_cast<int*>(sig + np);  // [np]
+    __shared__ int s_rot;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwarp = blockDim.x >> 5;
+    for (int e = tid; e < np * n; e += blockDim.x) {
+        const int j = e / n, i = e % n;
+        B[e] = j < n ? (double)R[(int64_t)j * ldr + i] : 0.0;
+    }
+    if (want_v)
+        for (int e = tid; e < np * np; e += blockDim.x) Vs[e] = (e / np == e % np) ? 1.0 : 0.0;
+    __syncthreads();
+    for (int sweep = 0; sweep < max_sweeps; ++sweep) {
+        // exact squared column norms at the start of every sweep
+        for (int j = warp; j < np; j += nwarp) {
+            double a = 0.0;
+            for (int i = lane; i < n; i += 32) a = fma(B[j * n + i], B[j * n + i], a);
+            a = warp_sum_d(a);
+            if (lane == 0) nrm[j] = a;
+        }
+        if (tid == 0) s_rot = 0;
+        __syncthreads();
+        // one HALF-warp per pair: all n/2 pairs of a round at once (32 warps)
+        const int hl = lane & 15, hw = 2 * warp + (lane >> 4), nhw = 2 * nwarp;
+        const unsigned hmask = (lane >> 4) ? 0xffff0000u : 0x0000ffffu;
+        for (int r = 0; r < np - 1; ++r) {
+            for (int k = hw; k < np / 2; k += nhw) {
+                int p = rr_player(k, r, np), q = rr_player(np - 1 - k, r, np);
+                if (p > q) {
+                    const int t = p;
+                    p = q;
+                    q = t;
+                }
+                double* bp = B + (size_t)p * n;
+                double* bq = B + (size_t)q * n;
+                double g = 0.0;
+                for (int i = hl; i < n; i += 16) g = fma(bp[i], bq[i], g);
+#pragma unroll
+                for (int o = 8; o > 0; o >>= 1) g += __shfl_xor_sync(hmask, g, o);
+                const double al = nrm[p], be = nrm[q];
+                if (g * g > tol2 * (al * be) && g != 0.0) {
+                    // rotate so that b_p' . b_q' = 0 (cot 2 theta = (be - al) / (2 g)):
+                    // t = tan theta = 2 g sign(d) / (|d| + sqrt(d^2 + 4 g^2)), d = be - al
+                    // The angle only steers convergence; the rotation applied is
+                    // exactly orthogonal whatever t is (c, s from t in fp64), so t
+                    // comes from fast fp32 arithmetic.
+                    const float df = (float)(be - al), gf = (float)g;
+                    const float tf = (df < 0.f ? -2.f * gf : 2.f * gf) *
+                                     __frcp_rn(fabsf(df) + sqrtf(fmaf(df, df, 4.f * gf * gf)));
+                    const double t = (double)tf;
+                    const double c = rsqrt(fma(t, t, 1.0)), s = c * t;
+                    for (int i = hl; i < n; i += 16) {
+                        const double x = bp[i], y = bq[i];
+                        bp[i] = c * x - s * y;
+                        bq[i] = s * x + c * y;
+                    }
+                    if (want_v) {
+                        double* vp = Vs + (size_t)p * np;
+                        double* vq = Vs + (size_t)q * np;
+                        for (int i = hl; i < np; i += 16) {
+                            const double x = vp[i], y = vq[i];
+                            vp[i] = c * x - s * y;
+                            vq[i] = s * x + c * y;
+                        }
+                    }
+                    if (hl == 0) {
+                        nrm[p] = al - t * g;
+                        nrm[q] = be + t * g;
+                        s_rot = 1;
+                    }
+                }
+            }
+            __syncthreads();
+        }
+        const int rot = s_rot;
+        __syncthreads();
+        if (!rot) break;
+    }
+    // sigma_j = ||b_j|| (exact), descending order (ties by index)
+    for (int j = warp; j < np; j += nwarp) {
+        double a = 0.0;
+        for (int i = lane; i < n; i += 32) a = fma(B[j * n + i], B[j * n + i], a);
+        a = warp_sum_d(a);
+        if (lane == 0) sig[j] = sqrt(a);
+    }
+    __syncthreads();
+    for (int j = tid; j < n; j += blockDim.x) {
+        int rk = 0;
+        for (int k = 0; k < n; ++k) rk += (sig[k] > sig[j]) || (sig[k] == sig[j] && k < j);
+        rank[j] = rk;
+    }
+    __syncthreads();
+    for (int e = tid; e < n * n; e += blockDim.x) {
+        const int j = e / n, i = e % n, rk = rank[j];
+        const double sj = sig[j];
+        U[(int64_t)rk * ldu + i] = (T)(sj > 0.0 ? B[j * n + i] / sj : 0.0);
+        if (want_v) V[(int64_t)rk * ldv + i] = (T)Vs[(size_t)j * np + i];
+        if (i == 0) sigma[rk] = (T)sj;
+    }
+}
+
+template <typename T>
+inline size_t jacobi_svd_smem(int n) {
+    const size_t np = (size_t)((n + 1) & ~1);
+    return sizeof(double) * (np * n + np * np + 2 * np) + sizeof(int) * np;
+}
+
+// W(n x n) = U diag(max(sigma - tau, 0)) V^T; one block per column k of W.
+template <typename T>
+__global__ void svt_core_kernel(int n, const T* __restrict__ U, int64_t ldu, const T* __restrict__ sigma,
+                                const T* __restrict__ V, int64_t ldv, T tau, T* __restrict__ W, int64_t ldw) {
+    const int k = blockIdx.x;
+    for (int i = threadIdx.x; i < n; i += blockDim.x) {
+        double acc = 0.0;
+        for (int j = 0; j < n; ++j) {
+            const double d = (double)sigma[j] - (double)tau;
+            if (d > 0.0) acc = fma((double)U[(int64_t)j * ldu + i] * d, (double)V[(int64_t)j * ldv + k], acc);
+        }
+        W[(int64_t)k * ldw + i] = (T)acc;
+    }
+}
+
+// W(n x n) = U diag(max(sigma - tau, 0) / sigma) U^T R  (== U diag(max(sigma - tau, 0)) V^T
+// for R = U diag(sigma) V^T: U^T R = diag(sigma) V^T; no V needed, and only
+// sigma_j > tau, hence no small sigma, is divided by).  One block per column k.
+template <typename T>
+__global__ void svt_core_r_kernel(int n, const T* __restrict__ U, int64_t ldu, const T* __restrict__ sigma,
+                                  const T* __restrict__ R, int64_t ldr, T tau, T* __restrict__ W, int64_t ldw) {
+    __shared__ double pk[kSvdMaxN];
+    const int k = blockIdx.x;
+    for (int j = threadIdx.x; j < n; j += blockDim.x) {  // pk_j = f(sigma_j) (U^T R)_jk
+        const double sj = (double)sigma[j], d = sj - (double)tau;
+        double acc = 0.0;
+        if (d > 0.0) {
+            for (int l = 0; l < n; ++l) acc = fma((double)U[(int64_t)j * ldu + l], (double)R[(int64_t)k * ldr + l], acc);
+            acc *= d / sj;
+        }
+        pk[j] = acc;
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < n; i += blockDim.x) {
+        double acc = 0.0;
+        for (int j = 0; j < n; ++j) acc = fma((double)U[(int64_t)j * ldu + i], pk[j], acc);
+        W[(int64_t)k * ldw + i] = (T)acc;
+    }
+}
+
+// C (m x n) = [W; 0], W n x n.
+template <typename T>
+__global__ void embed_top_kernel(int64_t m, int64_t n, const T* __restrict__ W, int64_t ldw, T* __restrict__ C,
+                                 int64_t ldc) {
+    const int64_t total = m * n;
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t j = e / m, i = e % m;
+        C[j * ldc + i] = i < n ? W[j * ldw + i] : T(0);
+    }
+}
+
+__device__ __forceinline__ double block_sum_d(double v, double* scr) {
+    v = warp_sum_d(v);
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    if (lane == 0) scr[warp] = v;
+    __syncthreads();
+    double t = 0.0;
+    if (threadIdx.x == 0)
+        for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += scr[w];
+    return t;
+}
+
+// Elementwise over m x n ([19]):
+//   S <- shrink(M - L + Y/mu, lambda/mu);  Y <- Y + mu (M - L - S);
+//   X <- M - S + Y/mu_next  (the next SVT input);  part[b] = sum (M - L - S)^2.
+template <typename T>
+__global__ void __launch_bounds__(256) rpca_update_kernel(int64_t m, int64_t n, const T* __restrict__ M, int64_t ldm,
+                                                          const T* __restrict__ L, int64_t ldl, T* __restrict__ S,
+                                                          int64_t lds, T* __restrict__ Y, int64_t ldy,
+                                                          T* __restrict__ X, int64_t ldx, T mu, T mu_next,
+                                                          T lambda, double* __restrict__ part) {
+    __shared__ double scr[8];
+    const T imu = T(1) / mu, imu_next = T(1) / mu_next, thr = lambda / mu;
+    double acc = 0.0;
+    const int64_t total = m * n;
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t j = e / m, i = e % m;
+        const T mv = M[j * ldm + i], lv = L[j * ldl + i], yv = Y[j * ldy + i];
+        const T t = mv - lv + yv * imu;
+        const T a = fabs(t) - thr;
+        const T sv = a > T(0) ? copysign(a, t) : T(0);
+        const T z = mv - lv - sv;
+        const T yn = yv + mu * z;
+        S[j * lds + i] = sv;
+        Y[j * ldy + i] = yn;
+        X[j * ldx + i] = mv - sv + yn * imu_next;
+        acc = fma((double)z, (double)z, acc);
+    }
+    const double b = block_sum_d(acc, scr);
+    if (threadIdx.x == 0) part[1 + blockIdx.x] = b;
+}
+
+// part[0] = sum of part[1..nb] in index order (deterministic).
+__global__ void sum_parts_kernel(int nb, double* part) {
+    __shared__ double scr[32];
+    double a = 0.0;
+    // fixed assignment of parts to threads and a fixed tree: deterministic
+    for (int b = threadIdx.x; b < nb; b += blockDim.x) a += part[1 + b];
+    const double t = block_sum_d(a, scr);
+    if (threadIdx.x == 0) part[0] = t;
+}
+
+// Start of the iteration: S = 0, Y = yscale M, X = M + Y / mu.
+template <typename T>
+__global__ void rpca_init_kernel(int64_t m, int64_t n, const T* __restrict__ M, int64_t ldm, T yscale,
+                                 T* __restrict__ S, int64_t lds, T* __restrict__ Y, int64_t ldy, T* __restrict__ X,
+                                 int64_t ldx, T mu) {
+    const int64_t total = m * n;
+    const T imu = T(1) / mu;
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t j = e / m, i = e % m;
+        const T mv = M[j * ldm + i];
+        const T yv = yscale * mv;
+        S[j * lds + i] = T(0);
+        Y[j * ldy + i] = yv;
+        X[j * ldx + i] = mv + yv * imu;
+    }
+}
+
+// out[0] = max |M_ij| (as the bits of a non-negative float: integer max is
+// order-independent, so the result is deterministic).
+template <typename T>
+__global__ void absmax_kernel(int64_t m, int64_t n, const T* __restrict__ M, int64_t ldm, T* out) {
+    __shared__ T scr[32];
+    T a = T(0);
+    const int64_t total = m * n;
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t j = e / m, i = e % m;
+        a = fmax(a, fabs(M[j * ldm + i]));
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) a = fmax(a, __shfl_xor_sync(0xffffffffu, a, o));
+    if ((threadIdx.x & 31) == 0) scr[threadIdx.x >> 5] = a;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int w = 1; w < (int)(blockDim.x >> 5); ++w) a = fmax(a, scr[w]);
+        if constexpr (sizeof(T) == 4)
+            atomicMax(reinterpret_cast<unsigned int*>(out), __float_as_uint(a));
+        else
+            atomicMax(reinterpret_cast<unsigned long long*>(out), (unsigned long long)__double_as_longlong(a));
+    }
+}
+
+}  // namespace caqr
