@@ -833,7 +833,11 @@ static int svd_small_impl(int64_t n, const T* R, int64_t ldr, T* U, int64_t ldu,
         // a pair counts as orthogonal at |b_p.b_q| <= tol ||b_p|| ||b_q||: U's
         // orthogonality is tol-level, far below the output precision's epsilon
         const double tol = sizeof(T) == 4 ? 1e-10 : 1e-15;
-        jacobi_svd_kernel<T><<<1, kSvdThreads, smem, s>>>((int)n, R, ldr, U, ldu, sigma, V, ldv, tol, 30);
+        static const int max_sweeps = [] {
+            const char* e = getenv("CAQR_SVD_SWEEPS");  // diagnostics: cap the Jacobi sweeps
+            return e ? std::max(1, atoi(e)) : 30;
+        }();
+        jacobi_svd_kernel<T><<<1, kSvdThreads, smem, s>>>((int)n, R, ldr, U, ldu, sigma, V, ldv, tol, max_sweeps);
         e = cudaGetLastError();
     }
     if (e != cudaSuccess) {

@@ -22,7 +22,7 @@
 
 namespace caqr {
 
-constexpr int kSvdMaxN = 112;     // 2 n^2 doubles in shared memory (B and V)
+constexpr int kSvdMaxN = 112;     // 2 n^2 doubles in shared memory (B and V); n/2 <= 64 half-warps
 constexpr int kSvdThreads = 1024;
 constexpr int kRpcaBlocks = 1024;  // partial sums of the residual (fixed grid)
 
@@ -70,16 +70,15 @@ jacobi_svd_kernel(int n, const T* __restrict__ R, int64_t ldr, T* __restrict__ U
         if (tid == 0) s_rot = 0;
         __syncthreads();
         // one HALF-warp per pair: all n/2 pairs of a round at once (32 warps)
-        const int hl = lane & 15, hw = 2 * warp + (lane >> 4), nhw = 2 * nwarp;
+        const int hl = lane & 15, hw = 2 * warp + (lane >> 4);
         const unsigned hmask = (lane >> 4) ? 0xffff0000u : 0x0000ffffu;
-        for (int r = 0; r < np - 1; ++r) {
-            for (int k = hw; k < np / 2; k += nhw) {
-                int p = rr_player(k, r, np), q = rr_player(np - 1 - k, r, np);
-                if (p > q) {
-                    const int t = p;
-                    p = q;
-                    q = t;
-                }
+        // (n <= 112: np/2 <= 56 pairs <= 64 half-warps, so each has at most one;
+        // its two players advance by the circle method: x -> x + 1, np-1 -> 1)
+        int pa = rr_player(hw, 0, np), pb = rr_player(np - 1 - hw, 0, np);
+        for (int r = 0; r < np - 1; ++r, pa = pa == 0 ? 0 : (pa == np - 1 ? 1 : pa + 1),
+                 pb = pb == np - 1 ? 1 : pb + 1) {
+            if (hw < np / 2) {
+                const int p = min(pa, pb), q = max(pa, pb);
                 double* bp = B + (size_t)p * n;
                 double* bq = B + (size_t)q * n;
                 double g = 0.0;
