@@ -1,4 +1,7 @@
 // panel_lpc.cuh -- "lane per column" Householder panel factorization.
+// EXPERIMENT (not used by libcaqr): measured by tools/lpc_bench.cu on a B200 at
+// 55k cycles per 256 x 32 panel vs 29k for the library's WB4 scheme (1 CTA),
+// so WB4 stays; kept as the record of that negative result.
 //
 // The paper's fastest apply kernel keeps each thread's data in registers and
 // does its reductions serially inside the thread ("register-file serial
@@ -19,7 +22,7 @@
 // Two CTA barriers and no shuffles per column.  Reflector heads (rows j < 32)
 // all sit in warp 0.
 #pragma once
-#include "tsqr_kernels.cuh"
+#include "../paper_conf_ipps_andersonbdk11_b200/csrc/tsqr_kernels.cuh"
 
 namespace caqr {
 
