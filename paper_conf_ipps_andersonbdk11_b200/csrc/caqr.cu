@@ -27,10 +27,11 @@ static thread_local int g_last_cuda_error = 0;
 // stream + host-computed algorithmic flops/bytes; see caqr_trace_begin) -------
 enum KernelId { K_PANEL_FACTOR = 0, K_PANEL_UPDATE = 1, K_EXTRACT_R = 2, K_SET_IDENTITY = 3,
                 K_TSQR_FUSED = 4, K_TSQR_SKINNY = 5, K_SVD_SMALL = 6, K_SVT_CORE = 7, K_EMBED_TOP = 8,
-                K_RPCA_UPDATE = 9, K_RPCA_INIT = 10, K_ABSMAX = 11, K_NUM = 12 };
+                K_RPCA_UPDATE = 9, K_RPCA_INIT = 10, K_ABSMAX = 11, K_CHAIN_UPDATE = 12, K_NUM = 13 };
 static const char* const kKernelNames[K_NUM] = {"panel_factor", "panel_update", "extract_r", "set_identity",
                                                 "tsqr_fused",   "tsqr_skinny",  "svd_small", "svt_core",
-                                                "embed_top",    "rpca_update",  "rpca_init", "absmax"};
+                                                "embed_top",    "rpca_update",  "rpca_init", "absmax",
+                                                "node_update"};
 struct Trace {
     std::mutex mu;
     bool on = false;
@@ -318,6 +319,55 @@ static int launch_update(const Geom& G, const T* A, const T* Tws, int level, int
     return 0;
 }
 
+// Q^T C / Q C node by node: one launch for every chain's tiles and panels
+// (level < 0) or for one whole tree level (node_update_kernel), instead of one
+// launch per (tile or level, panel).  CAQR_CHAIN_APPLY=0 restores the
+// per-(tile or level, panel) launches.
+static inline bool chain_apply_policy() {
+    const char* e = getenv("CAQR_CHAIN_APPLY");
+    return !(e && e[0] == '0');
+}
+
+template <typename T>
+static int launch_node_update(const Geom& G, const T* A, const T* Tws, int level, T* C, int64_t ldc,
+                              int64_t cfirst, int64_t ccount, int trans, cudaStream_t s) {
+    const int64_t nodes = level < 0 ? G.P : merges_at(G.P, level);
+    if (nodes <= 0 || ccount <= 0) return 0;
+    // tallest node: a [chain R; tile] step (<= 32 slot rows + b tile rows) or a
+    // merge (<= 32 + ncols rows)
+    const int rgmax = level < 0 ? (int)(G.K > 1 ? G.b + kPW : std::min<int64_t>(G.b, G.mrows))
+                                : (int)(kPW + std::min<int64_t>(G.ncols, G.b));
+    const size_t smem = panel_update_smem<T>(rgmax);
+    cudaError_t e = allow_smem(node_update_kernel<T, false>, smem);
+    double fl = 0, by = 0;
+    if (g_trace.on) {
+        for (int kt = 0; kt < (level < 0 ? G.K : 1); ++kt)
+            for (int p = 0; p < G.npan; ++p) {
+                double f1, b1;
+                trace_counts(G, level, p, kt, nodes, true, ccount, sizeof(T), &f1, &b1);
+                fl += f1;
+                by += b1;
+            }
+    }
+    TraceScope ts(level < 0 ? K_CHAIN_UPDATE : K_PANEL_UPDATE, fl, by, s);
+    if (e == cudaSuccess) {
+        // one CTA per (node, group of 32-column blocks): each node's V / T staged
+        // once per CTA, with >= 2 CTAs per SM when there are enough blocks
+        const int64_t nblk = ceil_div(ccount, 32);
+        const int64_t groups = std::max<int64_t>(1, std::min<int64_t>(nblk, (2 * num_sms()) / nodes));
+        const int64_t cpb = ceil_div(nblk, groups);
+        dim3 grid((unsigned)nodes, (unsigned)ceil_div(nblk, cpb));
+        node_update_kernel<T, false><<<grid, kThreads, smem, s>>>(G, A, Tws, level, C, ldc, cfirst, ccount, trans,
+                                                                  (int)cpb);
+        e = cudaGetLastError();
+    }
+    if (e != cudaSuccess) {
+        g_last_cuda_error = (int)e;
+        return CAQR_ERR_CUDA;
+    }
+    return 0;
+}
+
 // Phase profile of the fused kernel (diagnostics, CAQR_PROFILE=1).
 static unsigned long long* g_prof = nullptr;
 static unsigned long long* prof_buffer() {
@@ -588,6 +638,18 @@ static int apply_group(const Geom& G, const T* A, const T* Tws, bool do_leaves, 
                        bool mma = false) {
     int rc = 0;
     const int nl = tree_levels(G.P);
+    if (!mma && chain_apply_policy()) {  // one launch per tree level (+ one for the chains)
+        if (trans) {
+            if (do_leaves) rc = launch_node_update<T>(G, A, Tws, -1, C, ldc, cfirst, ccount, 1, s);
+            for (int lv = 0; lv < nl && !rc; ++lv)
+                rc = launch_node_update<T>(G, A, Tws, lv, C, ldc, cfirst, ccount, 1, s);
+        } else {
+            for (int lv = nl - 1; lv >= 0 && !rc; --lv)
+                rc = launch_node_update<T>(G, A, Tws, lv, C, ldc, cfirst, ccount, 0, s);
+            if (do_leaves && !rc) rc = launch_node_update<T>(G, A, Tws, -1, C, ldc, cfirst, ccount, 0, s);
+        }
+        return rc;
+    }
     if (trans) {
         if (do_leaves)
             for (int kt = 0; kt < G.K && !rc; ++kt)

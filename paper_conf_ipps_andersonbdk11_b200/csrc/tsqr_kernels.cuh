@@ -317,18 +317,24 @@ template <bool PAD>
 __device__ __forceinline__ void gemm2_mma(const Grp& G, const float* Vs, float* Cs, const float* W, int RGP,
                                           int R32);
 
-template <typename T, bool MMA = false>
-__global__ void __launch_bounds__(kThreads)
-panel_update_kernel(Geom g, const T* A, const T* __restrict__ Tws, int level, int p, int kt, T* C,
-                    int64_t ldc, int64_t cfirst, int64_t ccount, int trans, int cpb) {
+// One (node, panel p) of the implicit Q applied to column blocks [blk_beg,
+// blk_end) of C: C <- (I - V T V^T)^T C (trans) or (I - V T V^T) C, on the node's
+// gathered rows (the horizontal / tree updates).  A device routine
+// so that one launch can walk a whole chain (chain_update_kernel) as well as
+// one launch per (level, panel) (panel_update_kernel).
+template <typename T, bool MMA>
+__device__ __forceinline__ void update_node(const Geom& g, const T* A, const T* __restrict__ Tws, int level,
+                                            int64_t node, int p, int kt, T* C, int64_t ldc, int64_t cfirst,
+                                            int64_t ccount, int trans, int64_t blk_beg, int64_t blk_end,
+                                            unsigned char* smem_raw) {
     using V4 = typename Vec4<T>::type;
     constexpr int VN = Vec4<T>::n;
-    extern __shared__ __align__(16) unsigned char smem_raw[];
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int wp = min(kPW, g.ncols - 32 * p);
-    const NodeRows nr = node_rows(g, level, blockIdx.x, p, wp, kt);
+    const NodeRows nr = node_rows(g, level, node, p, wp, kt);
     const int RG = nr.n0 + nr.n1;
     if (RG == 0) return;
+    __syncthreads();  // a previous call's readers of the shared tiles are done
     const int R32 = (RG + 31) & ~31;
     const int RGP = smem_col_stride<T>(RG);
     T* Vs = reinterpret_cast<T*>(smem_raw);
@@ -392,9 +398,7 @@ panel_update_kernel(Geom g, const T* A, const T* __restrict__ Tws, int level, in
         for (int e = tid; e < kPW * kPW; e += kThreads)
             Tt[(e & 31) * kTS + (e >> 5)] = ((e & 31) < wp && (e >> 5) < wp) ? tb[e] : T(0);
     }
-    const int64_t nblk = (ccount + 31) / 32;
-    const int64_t blk_end = min(nblk, (int64_t)(blockIdx.y + 1) * cpb);
-    for (int64_t blk = (int64_t)blockIdx.y * cpb; blk < blk_end; ++blk) {
+    for (int64_t blk = blk_beg; blk < blk_end; ++blk) {
     cb0 = cfirst + 32 * blk;
     ncb = (int)(cfirst + ccount - cb0 < 32 ? cfirst + ccount - cb0 : 32);
     __syncthreads();  // the previous block's readers of Cs are done
@@ -525,6 +529,41 @@ panel_update_kernel(Geom g, const T* A, const T* __restrict__ Tws, int level, in
     }
     }
     }  // column blocks of this CTA
+}
+
+template <typename T, bool MMA = false>
+__global__ void __launch_bounds__(kThreads)
+panel_update_kernel(Geom g, const T* A, const T* __restrict__ Tws, int level, int p, int kt, T* C,
+                    int64_t ldc, int64_t cfirst, int64_t ccount, int trans, int cpb) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int64_t nblk = (ccount + 31) / 32;
+    const int64_t blk_beg = (int64_t)blockIdx.y * cpb, blk_end = min(nblk, blk_beg + cpb);
+    update_node<T, MMA>(g, A, Tws, level, blockIdx.x, p, kt, C, ldc, cfirst, ccount, trans, blk_beg, blk_end,
+                        smem_raw);
+}
+
+// Every step of node blockIdx.x in one launch.  level < 0: chain blockIdx.x --
+// Q^T applies tile 0 (the leaf) .. K-1, each panel 0 .. npan-1 (the order of
+// the factorization), Q the reverse; level >= 0: merge blockIdx.x of that tree
+// level, all its panels.  The nodes of one level touch disjoint rows, so no two
+// CTAs ever need each other's results: one launch per tree level (plus one for
+// all chains) instead of one per (level or tile, panel).
+template <typename T, bool MMA = false>
+__global__ void __launch_bounds__(kThreads)
+node_update_kernel(Geom g, const T* A, const T* __restrict__ Tws, int level, T* C, int64_t ldc, int64_t cfirst,
+                   int64_t ccount, int trans, int cpb) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int64_t node = blockIdx.x;
+    const int ntile = level < 0 ? (int)min(g.K, g.L - node * g.K) : 1;
+    const int64_t nblk = (ccount + 31) / 32;
+    const int64_t blk_beg = (int64_t)blockIdx.y * cpb, blk_end = min(nblk, blk_beg + cpb);
+    const int steps = ntile * g.npan;
+    for (int s = 0; s < steps; ++s) {
+        const int kt = trans ? s / g.npan : ntile - 1 - s / g.npan;
+        const int p = trans ? s % g.npan : g.npan - 1 - s % g.npan;
+        update_node<T, MMA>(g, A, Tws, level, node, p, kt, C, ldc, cfirst, ccount, trans, blk_beg, blk_end,
+                            smem_raw);
+    }
 }
 
 template <typename T>
