@@ -24,6 +24,7 @@ namespace caqr {
 
 constexpr int kSvdMaxN = 112;     // 2 n^2 doubles in shared memory (B and V); n/2 <= 64 half-warps
 constexpr int kSvdThreads = 1024;
+constexpr int kSvdRpl = (kSvdMaxN + 15) / 16;  // rows per lane of a half-warp
 constexpr int kRpcaBlocks = 1024;  // partial sums of the residual (fixed grid)
 
 __device__ __forceinline__ double warp_sum_d(double v) {
@@ -81,8 +82,21 @@ jacobi_svd_kernel(int n, const T* __restrict__ R, int64_t ldr, T* __restrict__ U
                 const int p = min(pa, pb), q = max(pa, pb);
                 double* bp = B + (size_t)p * n;
                 double* bq = B + (size_t)q * n;
-                double g = 0.0;
-                for (int i = hl; i < n; i += 16) g = fma(bp[i], bq[i], g);
+                // (rows hl + 16 t, t < 7: fully unrolled, every load issued up front)
+                double xp[kSvdRpl], xq[kSvdRpl];
+#pragma unroll
+                for (int t = 0; t < kSvdRpl; ++t) {
+                    const int i = hl + 16 * t;
+                    xp[t] = i < n ? bp[i] : 0.0;
+                    xq[t] = i < n ? bq[i] : 0.0;
+                }
+                double g = 0.0, g1 = 0.0;
+#pragma unroll
+                for (int t = 0; t < kSvdRpl; t += 2) {
+                    g = fma(xp[t], xq[t], g);
+                    if (t + 1 < kSvdRpl) g1 = fma(xp[t + 1], xq[t + 1], g1);
+                }
+                g += g1;
 #pragma unroll
                 for (int o = 8; o > 0; o >>= 1) g += __shfl_xor_sync(hmask, g, o);
                 const double al = nrm[p], be = nrm[q];
@@ -97,10 +111,13 @@ jacobi_svd_kernel(int n, const T* __restrict__ R, int64_t ldr, T* __restrict__ U
                                      __frcp_rn(fabsf(df) + sqrtf(fmaf(df, df, 4.f * gf * gf)));
                     const double t = (double)tf;
                     const double c = rsqrt(fma(t, t, 1.0)), s = c * t;
-                    for (int i = hl; i < n; i += 16) {
-                        const double x = bp[i], y = bq[i];
-                        bp[i] = c * x - s * y;
-                        bq[i] = s * x + c * y;
+#pragma unroll
+                    for (int t = 0; t < kSvdRpl; ++t) {
+                        const int i = hl + 16 * t;
+                        if (i < n) {
+                            bp[i] = c * xp[t] - s * xq[t];
+                            bq[i] = s * xp[t] + c * xq[t];
+                        }
                     }
                     if (want_v) {
                         double* vp = Vs + (size_t)p * np;
