@@ -101,6 +101,8 @@ static int make_plan(int64_t m, int64_t n, int dtype, const caqr_opts* o, int op
     // streaming kernel: one chain per warp, 8 warps per SM (148 SMs)
     const bool s16 = pl->skinny && n <= 8 && stream16_policy();
     pl->chain_target = pl->skinny ? (s16 ? 2 * kStreamChains : kStreamChains) : kChainTarget;
+    if (const char* e = getenv("CAQR_CHAIN_TARGET"))  // diagnostics: chains per group (tile sweep)
+        pl->chain_target = std::max<int64_t>(1, atoll(e));
     int64_t b = (o && o->leaf_rows > 0) ? o->leaf_rows
                                         : (pl->skinny ? (n <= 8 && !s16 ? 256 : 128)
                                                       : (nb <= kFusedLeaf ? kFusedLeaf : kMaxLeaf));
