@@ -335,6 +335,11 @@ __device__ __forceinline__ void update_node(const Geom& g, const T* A, const T* 
     const int RG = nr.n0 + nr.n1;
     if (RG == 0) return;
     __syncthreads();  // a previous call's readers of the shared tiles are done
+    // 16-byte C stores: C aligned, ldc % 4 == 0 and every gathered-row segment
+    // (R slots, tiles) starting on a multiple of 4 rows
+    const bool vec_p = sizeof(T) == 4 && (reinterpret_cast<uintptr_t>(C) % 16 == 0) && (ldc % 4 == 0) &&
+                       (g.row0 % 4 == 0) && (g.b % 4 == 0) && (g.bm % 4 == 0) && (nr.r0 % 4 == 0) &&
+                       (nr.r1 % 4 == 0) && (nr.n0 % 4 == 0);
     const int R32 = (RG + 31) & ~31;
     const int RGP = smem_col_stride<T>(RG);
     T* Vs = reinterpret_cast<T*>(smem_raw);
@@ -518,10 +523,18 @@ __device__ __forceinline__ void update_node(const Geom& g, const T* A, const T* 
                 for (int i = 0; i < 4; ++i) acc[i][c] = fma(-vr[i], wv, acc[i][c]);
             }
         }
+        const bool v4 = sizeof(T) == 4 && vec_p && r + 4 <= RG;  // rows r..r+3: one segment, 16-byte aligned
 #pragma unroll
         for (int c = 0; c < 8; ++c) {
             if (cbase + c >= ncb) break;
             T* ccol = C + (cb0 + cbase + c) * ldc;
+            if constexpr (sizeof(T) == 4) {
+                if (v4) {
+                    *reinterpret_cast<float4*>(ccol + gathered_row(nr, r)) =
+                        make_float4(acc[0][c], acc[1][c], acc[2][c], acc[3][c]);
+                    continue;
+                }
+            }
 #pragma unroll
             for (int i = 0; i < 4; ++i)
                 if (r + i < RG) ccol[gathered_row(nr, r + i)] = acc[i][c];
