@@ -407,7 +407,41 @@ __device__ __forceinline__ void update_node(const Geom& g, const T* A, const T* 
     cb0 = cfirst + 32 * blk;
     ncb = (int)(cfirst + ccount - cb0 < 32 ? cfirst + ccount - cb0 : 32);
     __syncthreads();  // the previous block's readers of Cs are done
-    stage(1);
+    if constexpr (sizeof(T) == 4) {
+        if (vec_p) {
+            // 16-byte loads of 4 consecutive gathered rows (one segment, aligned):
+            // a quarter of the load instructions, all issued before the stores
+            const int nq4 = R32 >> 2;  // <= 72
+            float4 b4[9];
+#pragma unroll
+            for (int u = 0; u < 9; ++u) {
+                const int e = tid + kThreads * u;
+                const int jj = e / nq4, r = 4 * (e - jj * nq4);
+                float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+                if (jj < ncb && r < RG) {
+                    const float* src = reinterpret_cast<const float*>(C) + (cb0 + jj) * ldc + gathered_row(nr, r);
+                    if (r + 4 <= RG) {
+                        v = __ldcg(reinterpret_cast<const float4*>(src));
+                    } else {
+                        v.x = src[0];
+                        if (r + 1 < RG) v.y = src[1];
+                        if (r + 2 < RG) v.z = src[2];
+                    }
+                }
+                b4[u] = v;
+            }
+#pragma unroll
+            for (int u = 0; u < 9; ++u) {
+                const int e = tid + kThreads * u;
+                const int jj = e / nq4, r = 4 * (e - jj * nq4);
+                if (jj < 32) *reinterpret_cast<float4*>(reinterpret_cast<float*>(Cs) + (size_t)jj * RGP + r) = b4[u];
+            }
+        } else {
+            stage(1);
+        }
+    } else {
+        stage(1);
+    }
     __syncthreads();
 
     if constexpr (MMA) {
