@@ -100,6 +100,7 @@ jacobi_svd_kernel(int n, const T* __restrict__ R, int64_t ldr, T* __restrict__ U
 #pragma unroll
                 for (int o = 8; o > 0; o >>= 1) g += __shfl_xor_sync(hmask, g, o);
                 const double al = nrm[p], be = nrm[q];
+                __syncwarp(hmask);  // every lane has read nrm before lane 0 rewrites it
                 if (g * g > tol2 * (al * be) && g != 0.0) {
                     // rotate so that b_p' . b_q' = 0 (cot 2 theta = (be - al) / (2 g)):
                     // t = tan theta = 2 g sign(d) / (|d| + sqrt(d^2 + 4 g^2)), d = be - al
