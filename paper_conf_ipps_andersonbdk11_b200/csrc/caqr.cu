@@ -17,6 +17,7 @@
 #include "tsqr_kernels.cuh"
 #include "tsqr_skinny.cuh"
 #include "rpca.cuh"
+#include "tsqr_stream_apply.cuh"
 #include "tsqr_stream.cuh"
 
 namespace caqr {
@@ -27,11 +28,12 @@ static thread_local int g_last_cuda_error = 0;
 // stream + host-computed algorithmic flops/bytes; see caqr_trace_begin) -------
 enum KernelId { K_PANEL_FACTOR = 0, K_PANEL_UPDATE = 1, K_EXTRACT_R = 2, K_SET_IDENTITY = 3,
                 K_TSQR_FUSED = 4, K_TSQR_SKINNY = 5, K_SVD_SMALL = 6, K_SVT_CORE = 7, K_EMBED_TOP = 8,
-                K_RPCA_UPDATE = 9, K_RPCA_INIT = 10, K_ABSMAX = 11, K_CHAIN_UPDATE = 12, K_NUM = 13 };
+                K_RPCA_UPDATE = 9, K_RPCA_INIT = 10, K_ABSMAX = 11, K_CHAIN_UPDATE = 12, K_STREAM_APPLY = 13,
+                K_NUM = 14 };
 static const char* const kKernelNames[K_NUM] = {"panel_factor", "panel_update", "extract_r", "set_identity",
                                                 "tsqr_fused",   "tsqr_skinny",  "svd_small", "svt_core",
                                                 "embed_top",    "rpca_update",  "rpca_init", "absmax",
-                                                "node_update"};
+                                                "node_update",  "stream_apply"};
 struct Trace {
     std::mutex mu;
     bool on = false;
@@ -370,6 +372,50 @@ static int launch_node_update(const Geom& G, const T* A, const T* Tws, int level
     return 0;
 }
 
+// Leaf level of Q^T C / Q C for skinny fp32 plans (one panel of <= 16 columns
+// on 256-row tiles for n <= 8, 128-row tiles for n <= 16): one warp per chain
+// (tsqr_stream_apply.cuh), C in groups of KC columns.  *done = false when the
+// plan does not qualify (node_update_kernel then runs).  CAQR_STREAM_APPLY=0
+// disables it.
+template <typename T>
+static int launch_stream_apply(const Geom& G, const T* A, const T* Tws, T* C, int64_t ldc, int64_t cfirst,
+                               int64_t ccount, int trans, cudaStream_t s, bool* done) {
+    *done = false;
+    if constexpr (sizeof(T) == 4) {
+        const char* env = getenv("CAQR_STREAM_APPLY");
+        if (env && env[0] == '0') return 0;
+        const bool nc8 = G.npan == 1 && G.ncols <= 8 && G.b == 256;
+        const bool nc16 = G.npan == 1 && G.ncols <= 16 && G.b == 128;
+        if (!nc8 && !nc16) return 0;
+        const int KC = nc8 ? 8 : 16;
+        const unsigned grid = (unsigned)ceil_div(G.P, kStreamApplyWarps);
+        cudaError_t e = cudaSuccess;
+        for (int64_t c0 = 0; c0 < ccount && e == cudaSuccess; c0 += KC) {
+            const int kk = (int)std::min<int64_t>(KC, ccount - c0);
+            T* Cg = C + (cfirst + c0) * ldc;
+            double fl = 0, by = 0;
+            if (g_trace.on) {
+                fl = 4.0 * (double)G.mrows * G.ncols * kk;
+                by = (double)G.mrows * (G.ncols + 2.0 * kk) * sizeof(T);
+            }
+            TraceScope ts(K_STREAM_APPLY, fl, by, s);
+            if (nc8)
+                stream_apply_chain_kernel<8, 8, 8><<<grid, 32 * kStreamApplyWarps, 0, s>>>(G, A, Tws, Cg, ldc, kk,
+                                                                                        trans);
+            else
+                stream_apply_chain_kernel<16, 16, 4><<<grid, 32 * kStreamApplyWarps, 0, s>>>(G, A, Tws, Cg, ldc,
+                                                                                          kk, trans);
+            e = cudaGetLastError();
+        }
+        if (e != cudaSuccess) {
+            g_last_cuda_error = (int)e;
+            return CAQR_ERR_CUDA;
+        }
+        *done = true;
+    }
+    return 0;
+}
+
 // Phase profile of the fused kernel (diagnostics, CAQR_PROFILE=1).
 static unsigned long long* g_prof = nullptr;
 static unsigned long long* prof_buffer() {
@@ -641,14 +687,20 @@ static int apply_group(const Geom& G, const T* A, const T* Tws, bool do_leaves, 
     int rc = 0;
     const int nl = tree_levels(G.P);
     if (!mma && chain_apply_policy()) {  // one launch per tree level (+ one for the chains)
+        auto leaves = [&](int tr) {
+            bool done = false;
+            int r = launch_stream_apply<T>(G, A, Tws, C, ldc, cfirst, ccount, tr, s, &done);
+            if (!r && !done) r = launch_node_update<T>(G, A, Tws, -1, C, ldc, cfirst, ccount, tr, s);
+            return r;
+        };
         if (trans) {
-            if (do_leaves) rc = launch_node_update<T>(G, A, Tws, -1, C, ldc, cfirst, ccount, 1, s);
+            if (do_leaves) rc = leaves(1);
             for (int lv = 0; lv < nl && !rc; ++lv)
                 rc = launch_node_update<T>(G, A, Tws, lv, C, ldc, cfirst, ccount, 1, s);
         } else {
             for (int lv = nl - 1; lv >= 0 && !rc; --lv)
                 rc = launch_node_update<T>(G, A, Tws, lv, C, ldc, cfirst, ccount, 0, s);
-            if (do_leaves && !rc) rc = launch_node_update<T>(G, A, Tws, -1, C, ldc, cfirst, ccount, 0, s);
+            if (do_leaves && !rc) rc = leaves(0);
         }
         return rc;
     }

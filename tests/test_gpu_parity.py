@@ -471,6 +471,7 @@ def test_node_update_matches_per_panel_launches(caqr, m, n, dtype, monkeypatch):
     """Q^T C / Q C / form_q with one launch per tree level (+ one for all chains)
     equal the per-(tile or level, panel) launches BITWISE: each node runs the
     same device routine in the same order; only the launch grouping differs."""
+    monkeypatch.setenv("CAQR_STREAM_APPLY", "0")  # (the warp-per-chain skinny apply sums in another order)
     tdt = torch.float32 if dtype == np.float32 else torch.float64
     A = workloads.gaussian(m, n, seed=5, dtype=dtype)
     C0 = workloads.gaussian(m, 3, seed=6, dtype=dtype)
@@ -494,3 +495,40 @@ def test_node_update_matches_per_panel_launches(caqr, m, n, dtype, monkeypatch):
     old = run()
     for a, b in zip(new, old):
         assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("m,n,k", [(4_000_000, 8, 8), (600_001, 5, 11), (1_000_003, 16, 16), (262_147, 12, 3)])
+def test_stream_apply_vs_node_update(caqr, m, n, k, monkeypatch):
+    """Skinny plans: the warp-per-chain leaf apply (tsqr_stream_apply.cuh) and
+    the CTA-per-node apply agree to rounding for Q^T C, Q C and form_q, and
+    Q^T Q = I, Q^T A = [R; 0] hold (C4-style bounds, BASELINE fp32)."""
+    bd = BOUNDS[np.float32]
+    A = workloads.gaussian(m, n, seed=k)
+    C0 = workloads.gaussian(m, k, seed=k + 1)
+    Ad = caqr.colmajor_empty(m, n)
+    Ad.copy_(torch.from_numpy(A))
+    R, ws = caqr.caqr_factor(Ad)
+
+    def run():
+        Q = caqr.caqr_form_q(Ad, ws)
+        C = caqr.colmajor_empty(m, k)
+        C.copy_(torch.from_numpy(C0))
+        caqr.caqr_apply_qt(Ad, ws, C)
+        D = caqr.colmajor_empty(m, k)
+        D.copy_(torch.from_numpy(C0))
+        caqr.caqr_apply_q(Ad, ws, D)
+        torch.cuda.synchronize()
+        return [t.cpu().double().numpy() for t in (Q, C, D)]
+
+    new = run()
+    monkeypatch.setenv("CAQR_STREAM_APPLY", "0")
+    old = run()
+    for a, b in zip(new, old):
+        assert np.linalg.norm(a - b) <= 1e-6 * np.linalg.norm(b)
+    Q = new[0]
+    R64 = R.cpu().double().numpy()
+    assert np.linalg.norm(Q.T @ Q - np.eye(n)) <= bd["orth"]
+    assert np.linalg.norm(A.astype(np.float64) - Q @ R64) / np.linalg.norm(A) <= bd["res"]
+    QtC = new[1]
+    Qt_ref = Q.T @ C0.astype(np.float64)
+    assert np.linalg.norm(QtC[:n] - Qt_ref) / np.linalg.norm(C0) <= bd["res"]
