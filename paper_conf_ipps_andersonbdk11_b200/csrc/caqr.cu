@@ -416,6 +416,38 @@ static int launch_stream_apply(const Geom& G, const T* A, const T* Tws, T* C, in
     return 0;
 }
 
+// One tree level of Q^T C / Q C for a single-panel group of <= 16 fp32
+// columns: one warp per merge (stream_apply_tree_kernel).  *done = false when
+// the group does not qualify.
+template <typename T>
+static int launch_stream_apply_tree(const Geom& G, const T* A, const T* Tws, int level, T* C, int64_t ldc,
+                                    int64_t cfirst, int64_t ccount, int trans, cudaStream_t s, bool* done) {
+    *done = false;
+    if constexpr (sizeof(T) == 4) {
+        const char* env = getenv("CAQR_STREAM_APPLY");
+        if (env && env[0] == '0') return 0;
+        if (G.npan != 1 || G.ncols > 16) return 0;
+        const int64_t nodes = merges_at(G.P, level);
+        *done = true;
+        if (nodes <= 0 || ccount <= 0) return 0;
+        const unsigned grid = (unsigned)ceil_div(nodes, kStreamApplyWarps);
+        TraceScope ts(K_STREAM_APPLY, 0.0, 0.0, s);
+        T* Cg = C + cfirst * ldc;
+        if (G.ncols <= 8)
+            stream_apply_tree_kernel<8><<<grid, 32 * kStreamApplyWarps, 0, s>>>(G, A, Tws, Cg, ldc, ccount, level,
+                                                                              trans);
+        else
+            stream_apply_tree_kernel<16><<<grid, 32 * kStreamApplyWarps, 0, s>>>(G, A, Tws, Cg, ldc, ccount, level,
+                                                                               trans);
+        const cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) {
+            g_last_cuda_error = (int)e;
+            return CAQR_ERR_CUDA;
+        }
+    }
+    return 0;
+}
+
 // Phase profile of the fused kernel (diagnostics, CAQR_PROFILE=1).
 static unsigned long long* g_prof = nullptr;
 static unsigned long long* prof_buffer() {
@@ -693,13 +725,17 @@ static int apply_group(const Geom& G, const T* A, const T* Tws, bool do_leaves, 
             if (!r && !done) r = launch_node_update<T>(G, A, Tws, -1, C, ldc, cfirst, ccount, tr, s);
             return r;
         };
+        auto level = [&](int lv, int tr) {
+            bool done = false;
+            int r = launch_stream_apply_tree<T>(G, A, Tws, lv, C, ldc, cfirst, ccount, tr, s, &done);
+            if (!r && !done) r = launch_node_update<T>(G, A, Tws, lv, C, ldc, cfirst, ccount, tr, s);
+            return r;
+        };
         if (trans) {
             if (do_leaves) rc = leaves(1);
-            for (int lv = 0; lv < nl && !rc; ++lv)
-                rc = launch_node_update<T>(G, A, Tws, lv, C, ldc, cfirst, ccount, 1, s);
+            for (int lv = 0; lv < nl && !rc; ++lv) rc = level(lv, 1);
         } else {
-            for (int lv = nl - 1; lv >= 0 && !rc; --lv)
-                rc = launch_node_update<T>(G, A, Tws, lv, C, ldc, cfirst, ccount, 0, s);
+            for (int lv = nl - 1; lv >= 0 && !rc; --lv) rc = level(lv, 0);
             if (do_leaves && !rc) rc = leaves(0);
         }
         return rc;

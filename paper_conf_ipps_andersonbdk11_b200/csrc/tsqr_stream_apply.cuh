@@ -141,4 +141,68 @@ stream_apply_chain_kernel(Geom g, const float* __restrict__ A, const float* __re
     }
 }
 
+
+// One tree level of Q^T C / Q C for a single-panel group of <= NC columns, one
+// WARP per merge ("apply_qt_tree"): lane cc < k holds column cc of
+// the C rows of both slots, V_2 (upper triangular, in R_b's slot) and T in
+// shared memory;  W = C_a + V_2^T C_b,  W <- T^T W (Q^T) or T W (Q),
+// C_a -= W,  C_b -= V_2 W.  k > 32 columns: the lanes loop over them.
+template <int NC>
+__global__ void __launch_bounds__(32 * kStreamApplyWarps)
+stream_apply_tree_kernel(Geom g, const float* __restrict__ A, const float* __restrict__ Tws, float* C, int64_t ldc,
+                         int64_t k, int level, int trans) {
+    __shared__ float s_V[kStreamApplyWarps][NC][NC + 1];
+    __shared__ float s_T[kStreamApplyWarps][NC][NC + 1];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t hl = int64_t(1) << level;
+    const int64_t nm = (g.P - 1 >= hl) ? (g.P - 1 - hl) / (2 * hl) + 1 : 0;
+    const int64_t node = (int64_t)blockIdx.x * kStreamApplyWarps + warp;
+    if (node >= nm) return;  // warp-uniform
+    const int wp = g.ncols;
+    const int64_t a = node << (level + 1), b = a + hl;
+    const int64_t ra = g.row0 + a * g.bm, rb = g.row0 + b * g.bm;
+    const int nbr = (int)min64(min64(g.b, g.mrows - b * g.bm), wp);  // rows of R_b's slot
+    const float* tb = Tws + ((g.L + b * g.K) * g.npan) * (kPW * kPW);
+    for (int e = lane; e < NC * NC; e += 32) {
+        const int i = e % NC, j = e / NC;
+        s_V[warp][i][j] = (i <= j && i < nbr && j < wp) ? __ldcg(A + (g.col0 + j) * g.lda + rb + i) : 0.f;
+        s_T[warp][i][j] = (i < wp && j < wp) ? __ldcg(tb + j * kPW + i) : 0.f;
+    }
+    __syncwarp();
+    for (int64_t cc = lane; cc < k; cc += 32) {
+        float ca[NC], cb[NC], w[NC];
+        float* colp = C + cc * ldc;
+#pragma unroll
+        for (int j = 0; j < NC; ++j) {
+            ca[j] = j < wp ? __ldcg(colp + ra + j) : 0.f;
+            cb[j] = j < nbr ? __ldcg(colp + rb + j) : 0.f;
+        }
+#pragma unroll
+        for (int j = 0; j < NC; ++j) {
+            float acc = ca[j];
+#pragma unroll
+            for (int i = 0; i <= j; ++i) acc = fmaf(s_V[warp][i][j], cb[i], acc);
+            w[j] = acc;
+        }
+        float w2[NC];
+#pragma unroll
+        for (int j = 0; j < NC; ++j) {
+            float acc = 0.f;
+#pragma unroll
+            for (int q = 0; q < NC; ++q) acc = fmaf(trans ? s_T[warp][q][j] : s_T[warp][j][q], w[q], acc);
+            w2[j] = acc;
+        }
+#pragma unroll
+        for (int j = 0; j < NC; ++j)
+            if (j < wp) colp[ra + j] = ca[j] - w2[j];
+#pragma unroll
+        for (int i = 0; i < NC; ++i) {
+            float acc = cb[i];
+#pragma unroll
+            for (int j = i; j < NC; ++j) acc = fmaf(-s_V[warp][i][j], w2[j], acc);
+            if (i < nbr) colp[rb + i] = acc;
+        }
+    }
+}
+
 }  // namespace caqr
