@@ -984,7 +984,7 @@ static int svd_small_impl(int64_t n, const T* R, int64_t ldr, T* U, int64_t ldu,
         TraceScope ts(K_SVD_SMALL, 0.0, 3.0 * n * n * sizeof(T), s);
         // a pair counts as orthogonal at |b_p.b_q| <= tol ||b_p|| ||b_q||: U's
         // orthogonality is tol-level, far below the output precision's epsilon
-        const double tol = sizeof(T) == 4 ? 1e-10 : 1e-15;
+        const double tol = sizeof(T) == 4 ? 1e-8 : 1e-15;
         static const int max_sweeps = [] {
             const char* e = getenv("CAQR_SVD_SWEEPS");  // diagnostics: cap the Jacobi sweeps
             return e ? std::max(1, atoi(e)) : 30;
