@@ -184,6 +184,28 @@ int caqr_dist_factor_f64(caqr_dist *h, int64_t m_local, int64_t n, double *A, in
                          void *cws, size_t cws_bytes, const caqr_opts *opts,
                          caqr_stream_t stream);
 
+/* ---- Least squares through the factorization -------------
+ * min ||A x - b||_2 for tall full-rank A, the use of QR the paper opens with
+ * (P:L86-92), with LAPACK xGELS semantics: B <- Q^T B, then rows 0..n-1 of B
+ * <- R^{-1} B[0:n] (the solution X, n x k); rows n..m-1 keep the residual's
+ * components (their column norms are the residual norms; S17: the rows
+ * themselves depend on the tree).
+ *   m, n, A, lda, ws, opts : exactly as passed to caqr_factor_* (R is read from
+ *   A's top n x n upper triangle)                    (info -1..-5 as apply_qt)
+ *   k, B, ldb              : as C / ldc of caqr_apply_qt (info -6, -7, -8).
+ * An exactly singular R gives Inf/NaN (no rank check, as xGELS). */
+int caqr_lstsq_f32(int64_t m, int64_t n, const float *A, int64_t lda, const void *ws, int64_t k,
+                   float *B, int64_t ldb, const caqr_opts *opts, caqr_stream_t stream);
+int caqr_lstsq_f64(int64_t m, int64_t n, const double *A, int64_t lda, const void *ws, int64_t k,
+                   double *B, int64_t ldb, const caqr_opts *opts, caqr_stream_t stream);
+/* B (n x k, ldb >= n) <- R^{-1} B, R upper triangular n x n (ldr >= n), on the
+ * device (one CTA per column, column-oriented back substitution; n <= 25,600
+ * fp64 / 51,200 fp32).  info: -1 n, -2 k, -3 R, -4 ldr, -5 B, -6 ldb. */
+int caqr_trsm_upper_f32(int64_t n, int64_t k, const float *R, int64_t ldr, float *B, int64_t ldb,
+                        caqr_stream_t stream);
+int caqr_trsm_upper_f64(int64_t n, int64_t k, const double *R, int64_t ldr, double *B, int64_t ldb,
+                        caqr_stream_t stream);
+
 /* ---- Application layer: SVD via QR and robust PCA (Sec. VI) -----------------
  * The paper's motivating workload: robust PCA of a video matrix
  * (one column per frame) by an alternating-directions method whose

@@ -99,6 +99,12 @@ def lib() -> ctypes.CDLL:
         L.caqr_dist_destroy.restype = None
         fl = ctypes.c_float
         for suf in ("f32", "f64"):
+            f = getattr(L, f"caqr_lstsq_{suf}")
+            f.argtypes = [i64, i64, vp, i64, vp, i64, vp, i64, op, vp]
+            f.restype = ip
+            f = getattr(L, f"caqr_trsm_upper_{suf}")
+            f.argtypes = [i64, i64, vp, i64, vp, i64, vp]
+            f.restype = ip
             f = getattr(L, f"caqr_svd_small_{suf}")
             f.argtypes = [i64, vp, i64, vp, i64, vp, vp, i64, vp]
             f.restype = ip
@@ -258,6 +264,22 @@ def caqr_form_q(A, ws, Q=None, n=None, opts=None, stream=None):
                                                  _stream(stream))
     _check(f"caqr_form_q_{suf}", info)
     return Q
+
+
+def caqr_lstsq(A, ws, B, n=None, opts=None, stream=None):
+    """Least squares (xGELS): B (m x k) <- Q^T B, then B[:n] <- R^{-1} B[:n] = argmin ||A X - B||.
+    Returns B; B[:n] is the solution, column norms of B[n:] the residual norms."""
+    return _apply("lstsq", A, ws, B, A.shape[1] if n is None else n, opts, stream)
+
+
+def caqr_trsm_upper(R, B, stream=None):
+    """B (n x k) <- R^{-1} B for upper-triangular R (n x n), on the device."""
+    code, suf = _dtype_code(R)
+    pr, ldr = _colmajor(R, "R")
+    pb, ldb = _colmajor(B, "B")
+    _check(f"caqr_trsm_upper_{suf}", getattr(lib(), f"caqr_trsm_upper_{suf}")(R.shape[0], B.shape[1], pr, ldr, pb,
+                                                                              ldb, _stream(stream)))
+    return B
 
 
 def caqr_combine_workspace_bytes(P: int, n: int, dtype: int = CAQR_F32) -> int:

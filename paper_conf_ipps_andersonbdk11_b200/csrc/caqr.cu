@@ -29,11 +29,11 @@ static thread_local int g_last_cuda_error = 0;
 enum KernelId { K_PANEL_FACTOR = 0, K_PANEL_UPDATE = 1, K_EXTRACT_R = 2, K_SET_IDENTITY = 3,
                 K_TSQR_FUSED = 4, K_TSQR_SKINNY = 5, K_SVD_SMALL = 6, K_SVT_CORE = 7, K_EMBED_TOP = 8,
                 K_RPCA_UPDATE = 9, K_RPCA_INIT = 10, K_ABSMAX = 11, K_CHAIN_UPDATE = 12, K_STREAM_APPLY = 13,
-                K_NUM = 14 };
+                K_TRSM = 14, K_NUM = 15 };
 static const char* const kKernelNames[K_NUM] = {"panel_factor", "panel_update", "extract_r", "set_identity",
                                                 "tsqr_fused",   "tsqr_skinny",  "svd_small", "svt_core",
                                                 "embed_top",    "rpca_update",  "rpca_init", "absmax",
-                                                "node_update",  "stream_apply"};
+                                                "node_update",  "stream_apply", "trsm_upper"};
 struct Trace {
     std::mutex mu;
     bool on = false;
@@ -1008,6 +1008,34 @@ static int launch_status() {
     return 0;
 }
 
+
+template <typename T>
+static int trsm_impl(int64_t n, int64_t k, const T* R, int64_t ldr, T* B, int64_t ldb, cudaStream_t s) {
+    if (n < 0) return -1;
+    if (k < 0) return -2;
+    if (ldr < std::max<int64_t>(1, n)) return -4;
+    if (ldb < std::max<int64_t>(1, n)) return -6;
+    if (n == 0 || k == 0) return 0;
+    if (!R) return -3;
+    if (!B) return -5;
+    const size_t smem = sizeof(T) * (size_t)n;
+    if (smem > 200 * 1024) return -1;
+    cudaError_t e = allow_smem(trsm_upper_kernel<T>, smem);
+    if (e == cudaSuccess) {
+        TraceScope ts(K_TRSM, (double)n * n * k, (double)n * n * sizeof(T) / 2 + 2.0 * n * k * sizeof(T), s);
+        for (int64_t c0 = 0; c0 < k && e == cudaSuccess; c0 += 65535) {
+            const unsigned g = (unsigned)std::min<int64_t>(65535, k - c0);
+            trsm_upper_kernel<T><<<g, 256, smem, s>>>(n, R, ldr, B + c0 * ldb, ldb);
+            e = cudaGetLastError();
+        }
+    }
+    if (e != cudaSuccess) {
+        g_last_cuda_error = (int)e;
+        return CAQR_ERR_CUDA;
+    }
+    return 0;
+}
+
 extern "C" {
 
 size_t caqr_workspace_bytes(int64_t m, int64_t n, int dtype, const caqr_opts* opts) {
@@ -1306,6 +1334,29 @@ int caqr_absmax_f32(int64_t m, int64_t n, const float* M, int64_t ldm, float* ou
     TraceScope ts(K_ABSMAX, 0.0, 4.0 * m * n, s);
     absmax_kernel<float><<<elem_grid(m * n, 256), 256, 0, s>>>(m, n, M, ldm, out);
     return launch_status();
+}
+
+
+// ---- least squares (xGELS through the CAQR factorization) -------------------
+int caqr_trsm_upper_f32(int64_t n, int64_t k, const float* R, int64_t ldr, float* B, int64_t ldb,
+                        caqr_stream_t stream) {
+    return trsm_impl<float>(n, k, R, ldr, B, ldb, (cudaStream_t)stream);
+}
+int caqr_trsm_upper_f64(int64_t n, int64_t k, const double* R, int64_t ldr, double* B, int64_t ldb,
+                        caqr_stream_t stream) {
+    return trsm_impl<double>(n, k, R, ldr, B, ldb, (cudaStream_t)stream);
+}
+int caqr_lstsq_f32(int64_t m, int64_t n, const float* A, int64_t lda, const void* ws, int64_t k, float* B,
+                   int64_t ldb, const caqr_opts* opts, caqr_stream_t stream) {
+    int rc = apply_impl<float>(m, n, A, lda, ws, k, B, ldb, opts, (cudaStream_t)stream, CAQR_F32, 1);
+    if (rc) return rc;
+    return trsm_impl<float>(n, k, A, lda, B, ldb, (cudaStream_t)stream);  // R: A's top n x n upper triangle
+}
+int caqr_lstsq_f64(int64_t m, int64_t n, const double* A, int64_t lda, const void* ws, int64_t k, double* B,
+                   int64_t ldb, const caqr_opts* opts, caqr_stream_t stream) {
+    int rc = apply_impl<double>(m, n, A, lda, ws, k, B, ldb, opts, (cudaStream_t)stream, CAQR_F64, 1);
+    if (rc) return rc;
+    return trsm_impl<double>(n, k, A, lda, B, ldb, (cudaStream_t)stream);
 }
 
 }  // extern "C"

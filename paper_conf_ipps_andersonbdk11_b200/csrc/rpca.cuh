@@ -314,4 +314,34 @@ __global__ void absmax_kernel(int64_t m, int64_t n, const T* __restrict__ M, int
     }
 }
 
+
+// X = R^{-1} B in place (R n x n upper triangular, B n x k), one CTA per
+// column of B: column-oriented back substitution with b in shared memory --
+// x_i = b_i / R_ii, then b_j -= R_ji x_i for j < i (coalesced over j).  The
+// triangular solve of least squares through QR (xGELS: x = R^{-1} (Q^T b)[0:n],
+// P:L86-92).
+template <typename T>
+__global__ void __launch_bounds__(256) trsm_upper_kernel(int64_t n, const T* __restrict__ R, int64_t ldr, T* B,
+                                                         int64_t ldb) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    T* b = reinterpret_cast<T*>(smem_raw);
+    __shared__ T s_x;
+    T* col = B + (int64_t)blockIdx.x * ldb;
+    for (int64_t j = threadIdx.x; j < n; j += blockDim.x) b[j] = col[j];
+    __syncthreads();
+    for (int64_t i = n - 1; i >= 0; --i) {
+        if (threadIdx.x == 0) {
+            const T xi = b[i] / R[i * ldr + i];
+            b[i] = xi;
+            s_x = xi;
+        }
+        __syncthreads();
+        const T xi = s_x;
+        const T* ri = R + i * ldr;
+        for (int64_t j = threadIdx.x; j < i; j += blockDim.x) b[j] -= ri[j] * xi;
+        __syncthreads();
+    }
+    for (int64_t j = threadIdx.x; j < n; j += blockDim.x) col[j] = b[j];
+}
+
 }  // namespace caqr
