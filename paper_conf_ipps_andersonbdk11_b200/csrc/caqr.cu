@@ -95,11 +95,16 @@ static int make_plan(int64_t m, int64_t n, int dtype, const caqr_opts* o, int op
     int64_t nb = (o && o->panel_cols > 0) ? o->panel_cols : (n <= kMaxGroup ? n : 64);
     if (nb > kMaxGroup) return -opt_pos;
     nb = std::max<int64_t>(1, std::min(nb, std::max<int64_t>(n, 1)));
-    // skinny fp32 panels (n <= 16, one group): one warp per task, 256-row (n <= 8)
-    // or 128-row (n <= 16) tiles, ~2,000 chains (see tsqr_skinny.cuh)
-    // (only for genuinely tall inputs: below ~256k rows the block kernel's
-    // fewer, larger tasks win, e.g. 4096 x 16: 0.13 ms vs 0.26 ms measured)
-    pl->skinny = dtype == CAQR_F32 && n <= 16 && nb >= n && m >= (int64_t(1) << 18);
+    // skinny fp32 panels (n <= 16, one group): one warp per chain, 256-row (n <= 8)
+    // or 128-row (n <= 16) tiles, ~1,100 chains (tsqr_stream.cuh).  With the
+    // arrival-counter tree it wins from m = 4096 up (measured 4096 x 16: 0.099 vs
+    // 0.139 ms for the block kernel; 65536 x 8: 0.078 vs 0.169; 200000 x 8: 0.095
+    // vs 0.207), so every m >= 1024 takes it.
+    static const int64_t skinny_min_m = [] {  // diagnostics: CAQR_SKINNY_MIN_M overrides the threshold
+        const char* e = getenv("CAQR_SKINNY_MIN_M");
+        return e ? (int64_t)atoll(e) : int64_t(1024);
+    }();
+    pl->skinny = dtype == CAQR_F32 && n <= 16 && nb >= n && m >= skinny_min_m;
     // streaming kernel: one chain per warp, 8 warps per SM (148 SMs)
     const bool s16 = pl->skinny && n <= 8 && stream16_policy();
     pl->chain_target = pl->skinny ? (s16 ? 2 * kStreamChains : kStreamChains) : kChainTarget;

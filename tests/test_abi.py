@@ -40,8 +40,13 @@ def test_workspace_bytes(L):
     def ws(L, npan, es):
         return 2 * L * npan * 1024 * es + -(-(32 + L * npan) * 4 // 256) * 256
     # default tile height 224 (n <= 224): 4096 rows -> 19 tiles, 1M rows -> 4465 tiles;
-    # skinny fp32 (n <= 16, m >= 2^18: warp-per-task kernel) uses 256/128-row tiles
-    assert caqr.caqr_workspace_bytes(4096, 16) == ws(19, 1, 4)
+    # skinny fp32 (n <= 16, m >= 1024: the warp-per-chain streaming kernel) uses
+    # 256 (n <= 8) / 128-row tiles and a cross-CTA exchange area in the flag
+    # area: 64 ints + one n x n R per CTA of 8 chains (32-int aligned) + 16
+    # counters per CTA: 4096 x 16 -> 32 tiles, 4 CTAs
+    nct = 4
+    sync = max(32 + 32, 64 + ((nct * 16 * 16 + 31) & ~31) + 16 * nct)
+    assert caqr.caqr_workspace_bytes(4096, 16) == 2 * 32 * 1024 * 4 + -(-sync * 4 // 256) * 256
     assert caqr.caqr_workspace_bytes(4096, 16, caqr.CAQR_F64) == ws(19, 1, 8)
     assert caqr.caqr_workspace_bytes(1_000_000, 192) == ws(4465, 6, 4)
     assert caqr.caqr_workspace_bytes(4096, 16, 0, caqr.make_opts(leaf_rows=256)) == ws(16, 1, 4)
