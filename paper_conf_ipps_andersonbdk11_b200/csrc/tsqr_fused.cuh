@@ -1049,11 +1049,17 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
         for (int kt = 0; kt < ntile; ++kt)
         for (int p = 0; p < g.npan; ++p) {
             const int wp = min(kPW, g.ncols - 32 * p);
-            if (level >= 0 && threadIdx.x == 0) {  // children's panel p must be final
+            // A slot's panel flag goes through 2v-1 ("panel p factored: its R rows
+            // of panel p's columns are final") and 2v ("panel p's trailing update
+            // done") for the node of version v that last writes it.  A merge
+            // factors its panel p once both children are factored, and updates
+            // its trailing columns once both are done: the factorization
+            // overlaps the children's trailing updates.
+            if (level >= 0 && threadIdx.x == 0) {
                 const int* fa = flags + slot_a * g.npan + p;
                 const int* fb = flags + slot_b * g.npan + p;
-                while (ld_acquire(fa) < ver_a) __nanosleep(64);
-                while (ld_acquire(fb) < ver_b) __nanosleep(64);
+                while (ld_acquire(fa) < 2 * ver_a - 1) __nanosleep(64);
+                while (ld_acquire(fb) < 2 * ver_b - 1) __nanosleep(64);
             }
             __syncthreads();
             CAQR_PROF(1);
@@ -1111,6 +1117,20 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
                     tb[e] = Tt[r * kTS + c];
                 }
             }
+            // wait for the children's trailing updates before touching later
+            // columns, then publish "factored" (the stored R / V of panel p are in A)
+            __threadfence();
+            __syncthreads();
+            if (threadIdx.x == 0) {
+                if (level >= 0) {  // (before this node's own publish on slot a: flags only grow)
+                    const int* fa = flags + slot_a * g.npan + p;
+                    const int* fb = flags + slot_b * g.npan + p;
+                    while (ld_acquire(fa) < 2 * ver_a) __nanosleep(64);
+                    while (ld_acquire(fb) < 2 * ver_b) __nanosleep(64);
+                }
+                if (kt == ntile - 1) st_release(flags + slot_a * g.npan + p, 2 * (level < 0 ? 1 : my_ver) - 1);
+            }
+            __syncthreads();
             CAQR_PROF(5);
             // ---- trailing columns of this node, 32 at a time -------------------
             // (the block holding the NEXT panel's columns goes last, so that
@@ -1140,8 +1160,8 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
             // ---- publish ----------------------------------------------------------
             __threadfence();
             __syncthreads();
-            if (threadIdx.x == 0 && kt == ntile - 1)  // the slot's R rows of panel p are final
-                st_release(flags + slot_a * g.npan + p, level < 0 ? 1 : my_ver);
+            if (threadIdx.x == 0 && kt == ntile - 1)  // panel p's trailing update done
+                st_release(flags + slot_a * g.npan + p, 2 * (level < 0 ? 1 : my_ver));
             CAQR_PROF(9);
         }
     }
