@@ -156,6 +156,13 @@ int caqr_combine_apply_f32(int P, int64_t n, const float *Rstack, int64_t ld, co
 int caqr_combine_apply_f64(int P, int64_t n, const double *Rstack, int64_t ld, const void *ws,
                            int trans, int64_t k, double *C, int64_t ldc, caqr_stream_t stream);
 
+/* Q (m x n, ldq >= m) = [I_n; 0]: the start of an explicit Q (caqr_form_q does
+ * it internally); used with caqr_combine_apply / caqr_apply_q to form the rows
+ * of a row-sharded factorization's Q on each rank.
+ * info: -1 m, -2 n (0 <= n <= m), -3 Q, -4 ldq. */
+int caqr_set_identity_f32(int64_t m, int64_t n, float *Q, int64_t ldq, caqr_stream_t stream);
+int caqr_set_identity_f64(int64_t m, int64_t n, double *Q, int64_t ldq, caqr_stream_t stream);
+
 /* ---- Multi-GPU row-sharded TSQR over NCCL (one process per GPU) -----------
  * caqr_dist_create: nccl_unique_id = the 128-byte ncclUniqueId made by rank 0
  * and broadcast by the caller (e.g. through torch.distributed).  The handle owns

@@ -102,6 +102,9 @@ def lib() -> ctypes.CDLL:
             f = getattr(L, f"caqr_lstsq_{suf}")
             f.argtypes = [i64, i64, vp, i64, vp, i64, vp, i64, op, vp]
             f.restype = ip
+            f = getattr(L, f"caqr_set_identity_{suf}")
+            f.argtypes = [i64, i64, vp, i64, vp]
+            f.restype = ip
             f = getattr(L, f"caqr_trsm_upper_{suf}")
             f.argtypes = [i64, i64, vp, i64, vp, i64, vp]
             f.restype = ip
@@ -270,6 +273,15 @@ def caqr_lstsq(A, ws, B, n=None, opts=None, stream=None):
     """Least squares (xGELS): B (m x k) <- Q^T B, then B[:n] <- R^{-1} B[:n] = argmin ||A X - B||.
     Returns B; B[:n] is the solution, column norms of B[n:] the residual norms."""
     return _apply("lstsq", A, ws, B, A.shape[1] if n is None else n, opts, stream)
+
+
+def caqr_set_identity(Q, stream=None):
+    """Q (m x n) = [I_n; 0] on the device."""
+    code, suf = _dtype_code(Q)
+    pq, ldq = _colmajor(Q, "Q")
+    _check(f"caqr_set_identity_{suf}", getattr(lib(), f"caqr_set_identity_{suf}")(Q.shape[0], Q.shape[1], pq, ldq,
+                                                                                  _stream(stream)))
+    return Q
 
 
 def caqr_trsm_upper(R, B, stream=None):

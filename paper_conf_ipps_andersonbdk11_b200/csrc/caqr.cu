@@ -1041,6 +1041,19 @@ static int trsm_impl(int64_t n, int64_t k, const T* R, int64_t ldr, T* B, int64_
     return 0;
 }
 
+// ---- [I_n; 0] -------------------------------------------------------------
+template <typename T>
+static int set_identity_impl(int64_t m, int64_t n, T* Q, int64_t ldq, cudaStream_t s) {
+    if (m < 0) return -1;
+    if (n < 0 || n > m) return -2;
+    if (ldq < std::max<int64_t>(1, m)) return -4;
+    if (m == 0 || n == 0) return 0;
+    if (!Q) return -3;
+    dim3 grid((unsigned)std::min<int64_t>(ceil_div(m, 256), 1024), (unsigned)n);
+    TraceScope ts(K_SET_IDENTITY, 0.0, (double)m * n * sizeof(T), s);
+    set_identity_kernel<T><<<grid, 256, 0, s>>>(m, n, Q, ldq);
+    return launch_status();
+}
 extern "C" {
 
 size_t caqr_workspace_bytes(int64_t m, int64_t n, int dtype, const caqr_opts* opts) {
@@ -1362,6 +1375,14 @@ int caqr_lstsq_f64(int64_t m, int64_t n, const double* A, int64_t lda, const voi
     int rc = apply_impl<double>(m, n, A, lda, ws, k, B, ldb, opts, (cudaStream_t)stream, CAQR_F64, 1);
     if (rc) return rc;
     return trsm_impl<double>(n, k, A, lda, B, ldb, (cudaStream_t)stream);
+}
+
+
+int caqr_set_identity_f32(int64_t m, int64_t n, float* Q, int64_t ldq, caqr_stream_t stream) {
+    return set_identity_impl<float>(m, n, Q, ldq, (cudaStream_t)stream);
+}
+int caqr_set_identity_f64(int64_t m, int64_t n, double* Q, int64_t ldq, caqr_stream_t stream) {
+    return set_identity_impl<double>(m, n, Q, ldq, (cudaStream_t)stream);
 }
 
 }  // extern "C"

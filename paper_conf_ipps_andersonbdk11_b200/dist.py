@@ -50,6 +50,29 @@ def allgather_r(R_local, group=None):
     return torch.cat(parts, dim=0)
 
 
+def local_form_q(A_local, ws, gather, cws, rank: int, world: int, opts=None, stream=None):
+    """Rows of the global thin Q held by rank `rank` (the
+    explicit basis of a row-sharded matrix, e.g. an s-step Krylov basis).
+
+    With A_p = Q_p R_p locally and [R_1; ...; R_P] = Q_c R (the combine), the
+    global factor is A = diag(Q_1 ... Q_P) Q_c R, so rank p's rows of Q are
+    Q_p Q_c[p n:(p+1) n, :] = Q_p_full [Q_c,p; 0].  Every rank forms the small
+    Q_c (P n x n) from the combine it already holds (identical bits on every
+    rank) and applies its local Q: no communication beyond the factor's
+    all-gather.  All steps are libcaqr kernels."""
+    from . import caqr
+
+    m, n = A_local.shape
+    Qc = caqr.colmajor_empty(world * n, n, A_local.dtype, A_local.device)
+    caqr.caqr_set_identity(Qc, stream=stream)
+    caqr.caqr_combine_apply(gather, world, cws, Qc, trans=False, stream=stream)
+    Q = caqr.colmajor_empty(m, n, A_local.dtype, A_local.device)
+    caqr.caqr_set_identity(Q, stream=stream)  # then overwrite the top n x n with Q_c,p
+    Q[:n].copy_(Qc[rank * n:(rank + 1) * n])
+    caqr.caqr_apply_q(A_local, ws, Q, opts=opts, stream=stream)
+    return Q
+
+
 class DistTSQR:
     """NCCL communicator owned by libcaqr (caqr_dist_create) for the ranks of a
     torch.distributed group; `factor` runs caqr_dist_factor_* on a local shard."""
@@ -95,6 +118,10 @@ class DistTSQR:
             cws.data_ptr(), cws.numel(), c._optp(opts), c._stream(stream))
         c._check(f"caqr_dist_factor_{suf}", info)
         return R, ws, gather, cws
+
+    def form_q(self, A_local, ws, gather, cws, opts=None, stream=None):
+        """This rank's rows of the global thin Q (after ``factor``)."""
+        return local_form_q(A_local, ws, gather, cws, self.rank, self.world, opts=opts, stream=stream)
 
     def close(self):
         if getattr(self, "handle", None) is not None:

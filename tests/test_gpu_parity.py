@@ -532,3 +532,38 @@ def test_stream_apply_vs_node_update(caqr, m, n, k, monkeypatch):
     QtC = new[1]
     Qt_ref = Q.T @ C0.astype(np.float64)
     assert np.linalg.norm(QtC[:n] - Qt_ref) / np.linalg.norm(C0) <= bd["res"]
+
+
+@pytest.mark.parametrize("m,n,P,dtype", [(4_000_000, 8, 4, np.float32), (200_000, 48, 3, np.float32),
+                                         (60_000, 40, 8, np.float64)])
+def test_sharded_form_q_emulated(caqr, m, n, P, dtype):
+    """The row-sharded explicit Q (dist.local_form_q: e.g. the
+    s-step Krylov basis across GPUs), emulated on one GPU: each shard factored
+    on its own, the stacked R's combined, then every shard's rows of Q formed
+    from the combine's Q_c and the local Q.  Stacked, they are the thin Q of
+    the whole matrix: Q^T Q = I, A = Q R, R against the oracle."""
+    from paper_conf_ipps_andersonbdk11_b200 import dist as cdist
+
+    tdt = torch.float32 if dtype == np.float32 else torch.float64
+    bd = BOUNDS[dtype]
+    A = workloads.gaussian(m, n, seed=P, dtype=dtype)
+    gather = caqr.colmajor_empty(P * n, n, tdt)
+    shards = []
+    for p in range(P):
+        s0, rows = cdist.shard_rows(m, P, p)
+        Ap = caqr.colmajor_empty(rows, n, tdt)
+        Ap.copy_(torch.from_numpy(A[s0:s0 + rows]))
+        Rp, wsp = caqr.caqr_factor(Ap)
+        gather[p * n:(p + 1) * n].copy_(Rp)
+        shards.append((Ap, wsp))
+    R, cws = caqr.caqr_combine(gather, P)
+    Q = np.concatenate([cdist.local_form_q(Ap, wsp, gather, cws, p, P).cpu().double().numpy()
+                        for p, (Ap, wsp) in enumerate(shards)])
+    R = R.cpu().double().numpy()
+    A64 = A.astype(np.float64)
+    assert np.linalg.norm(Q.T @ Q - np.eye(n)) <= bd["orth"]
+    assert np.linalg.norm(A64 - Q @ R) / np.linalg.norm(A64) <= bd["res"]
+    rows = min(m, 300_000)
+    if rows == m:
+        Ro = oracle.normalize_signs(oracle.qr(A64, want_q=False, acc=bd["acc"]))
+        assert np.linalg.norm(oracle.normalize_signs(R) - Ro) / np.linalg.norm(Ro) <= bd["r"]
