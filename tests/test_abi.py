@@ -96,3 +96,49 @@ def test_info_codes_without_gpu(L):
     assert c(0, 4, vp(8), 4, vp(8), 4, vp(8), 1 << 20, null) == -1
     assert c(2, 300, vp(8), 600, vp(8), 300, vp(8), 1 << 30, null) == -2
     assert L.caqr_strerror(-3) and L.caqr_strerror(1)
+
+
+def test_info_codes_application_layer_without_gpu(L):
+    """The f1 / f4 entry points validate their arguments (LAPACK info) before any
+    CUDA call: robust-PCA kernels, small SVD, least squares, triangular solve."""
+    vp = ctypes.c_void_p
+    null = None
+    one = vp(8)
+    # caqr_svd_small_f32(n, R, ldr, U, ldu, sigma, V, ldv, stream)
+    s = L.caqr_svd_small_f32
+    assert s(113, one, 113, one, 113, one, one, 113, null) == -1  # n > 112
+    assert s(-1, one, 1, one, 1, one, one, 1, null) == -1
+    assert s(8, one, 7, one, 8, one, one, 8, null) == -3
+    assert s(8, one, 8, one, 7, one, one, 8, null) == -5
+    assert s(8, one, 8, one, 8, one, one, 7, null) == -8
+    assert s(8, null, 8, one, 8, one, one, 8, null) == -2
+    assert s(8, one, 8, one, 8, null, one, 8, null) == -6
+    assert s(0, null, 1, null, 1, null, null, 1, null) == 0  # quick return
+    # caqr_svt_core_f32(n, U, ldu, sigma, V, ldv, tau, W, ldw, stream)
+    t = L.caqr_svt_core_f32
+    assert t(4, one, 4, one, one, 4, 1.0, one, 3, null) == -9
+    assert t(4, one, 4, null, one, 4, 1.0, one, 4, null) == -4
+    # caqr_rpca_update_f32(m, n, M, ldm, L, ldl, S, lds, Y, ldy, X, ldx, mu, mu_next, lambda, resid, stream)
+    u = L.caqr_rpca_update_f32
+    assert u(4, 2, one, 4, one, 4, one, 4, one, 4, one, 4, 0.0, 1.0, 0.1, one, null) == -13
+    assert u(4, 2, one, 4, one, 4, one, 4, one, 4, one, 4, 1.0, -1.0, 0.1, one, null) == -14
+    assert u(4, 2, one, 4, one, 4, one, 4, one, 4, one, 4, 1.0, 1.0, -0.1, one, null) == -15
+    assert u(4, 2, one, 4, one, 4, one, 4, one, 4, one, 4, 1.0, 1.0, 0.1, null, null) == -16
+    assert u(4, 2, one, 4, one, 3, one, 4, one, 4, one, 4, 1.0, 1.0, 0.1, one, null) == -6
+    assert u(4, 2, one, 4, null, 4, one, 4, one, 4, one, 4, 1.0, 1.0, 0.1, one, null) == -5
+    # caqr_embed_top_f32(m, n, W, ldw, C, ldc, stream)
+    e = L.caqr_embed_top_f32
+    assert e(4, 5, one, 5, one, 4, null) == -2 and e(4, 2, one, 2, one, 3, null) == -6
+    # caqr_trsm_upper_f32(n, k, R, ldr, B, ldb, stream)
+    r = L.caqr_trsm_upper_f32
+    assert r(-1, 1, one, 1, one, 1, null) == -1 and r(4, -1, one, 4, one, 4, null) == -2
+    assert r(4, 1, one, 3, one, 4, null) == -4 and r(4, 1, one, 4, one, 3, null) == -6
+    assert r(4, 1, null, 4, one, 4, null) == -3 and r(0, 3, null, 1, null, 1, null) == 0
+    # caqr_lstsq_f32(m, n, A, lda, ws, k, B, ldb, opts, stream): apply_qt's numbering
+    q = L.caqr_lstsq_f32
+    assert q(4, 5, one, 4, one, 1, one, 4, null, null) == -2
+    assert q(4, 2, one, 4, one, -1, one, 4, null, null) == -6
+    assert q(4, 2, one, 4, one, 1, one, 3, null, null) == -8
+    # caqr_set_identity_f32(m, n, Q, ldq, stream)
+    i = L.caqr_set_identity_f32
+    assert i(4, 5, one, 4, null) == -2 and i(4, 2, one, 3, null) == -4 and i(4, 2, null, 4, null) == -3
