@@ -25,6 +25,7 @@ namespace caqr {
 constexpr int kSvdMaxN = 112;     // 2 n^2 doubles in shared memory (B and V); n/2 <= 64 half-warps
 constexpr int kSvdThreads = 1024;
 constexpr int kSvdRpl = (kSvdMaxN + 15) / 16;  // rows per lane of a half-warp
+constexpr int kSvdLd = 16 * kSvdRpl;           // padded column length of B
 constexpr int kRpcaBlocks = 1024;  // partial sums of the residual (fixed grid)
 
 __device__ __forceinline__ double warp_sum_d(double v) {
@@ -46,16 +47,18 @@ jacobi_svd_kernel(int n, const T* __restrict__ R, int64_t ldr, T* __restrict__ U
     const bool want_v = V != nullptr;
     extern __shared__ __align__(16) double sm[];
     const int np = (n + 1) & ~1;  // an odd n gets a zero column (never rotated)
-    double* B = sm;               // [np][n]  column j at B + j * n
-    double* Vs = B + (size_t)np * n;  // [np][np]
+    // columns padded with zero rows to kSvdLd = 16 * kSvdRpl: the half-warp
+    // loops need no bounds (a rotation keeps zero rows zero)
+    double* B = sm;                          // [np][kSvdLd]  column j at B + j * kSvdLd
+    double* Vs = B + (size_t)np * kSvdLd;    // [np][np]
     double* nrm = Vs + (size_t)np * np;  // [np]
     double* sig = nrm + np;              // [np]
     int* rank = reinterpret_cast<int*>(sig + np);  // [np]
     __shared__ int s_rot;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwarp = blockDim.x >> 5;
-    for (int e = tid; e < np * n; e += blockDim.x) {
-        const int j = e / n, i = e % n;
-        B[e] = j < n ? (double)R[(int64_t)j * ldr + i] : 0.0;
+    for (int e = tid; e < np * kSvdLd; e += blockDim.x) {
+        const int j = e / kSvdLd, i = e % kSvdLd;
+        B[e] = (j < n && i < n) ? (double)R[(int64_t)j * ldr + i] : 0.0;
     }
     if (want_v)
         for (int e = tid; e < np * np; e += blockDim.x) Vs[e] = (e / np == e % np) ? 1.0 : 0.0;
@@ -64,7 +67,7 @@ jacobi_svd_kernel(int n, const T* __restrict__ R, int64_t ldr, T* __restrict__ U
         // exact squared column norms at the start of every sweep
         for (int j = warp; j < np; j += nwarp) {
             double a = 0.0;
-            for (int i = lane; i < n; i += 32) a = fma(B[j * n + i], B[j * n + i], a);
+            for (int i = lane; i < n; i += 32) a = fma(B[j * kSvdLd + i], B[j * kSvdLd + i], a);
             a = warp_sum_d(a);
             if (lane == 0) nrm[j] = a;
         }
@@ -80,15 +83,14 @@ jacobi_svd_kernel(int n, const T* __restrict__ R, int64_t ldr, T* __restrict__ U
                  pb = pb == np - 1 ? 1 : pb + 1) {
             if (hw < np / 2) {
                 const int p = min(pa, pb), q = max(pa, pb);
-                double* bp = B + (size_t)p * n;
-                double* bq = B + (size_t)q * n;
+                double* bp = B + p * kSvdLd + hl;
+                double* bq = B + q * kSvdLd + hl;
                 // (rows hl + 16 t, t < 7: fully unrolled, every load issued up front)
                 double xp[kSvdRpl], xq[kSvdRpl];
 #pragma unroll
                 for (int t = 0; t < kSvdRpl; ++t) {
-                    const int i = hl + 16 * t;
-                    xp[t] = i < n ? bp[i] : 0.0;
-                    xq[t] = i < n ? bq[i] : 0.0;
+                    xp[t] = bp[16 * t];
+                    xq[t] = bq[16 * t];
                 }
                 double g = 0.0, g1 = 0.0;
 #pragma unroll
@@ -114,11 +116,8 @@ jacobi_svd_kernel(int n, const T* __restrict__ R, int64_t ldr, T* __restrict__ U
                     const double c = rsqrt(fma(t, t, 1.0)), s = c * t;
 #pragma unroll
                     for (int t = 0; t < kSvdRpl; ++t) {
-                        const int i = hl + 16 * t;
-                        if (i < n) {
-                            bp[i] = c * xp[t] - s * xq[t];
-                            bq[i] = s * xp[t] + c * xq[t];
-                        }
+                        bp[16 * t] = c * xp[t] - s * xq[t];
+                        bq[16 * t] = s * xp[t] + c * xq[t];
                     }
                     if (want_v) {
                         double* vp = Vs + (size_t)p * np;
@@ -145,7 +144,7 @@ jacobi_svd_kernel(int n, const T* __restrict__ R, int64_t ldr, T* __restrict__ U
     // sigma_j = ||b_j|| (exact), descending order (ties by index)
     for (int j = warp; j < np; j += nwarp) {
         double a = 0.0;
-        for (int i = lane; i < n; i += 32) a = fma(B[j * n + i], B[j * n + i], a);
+        for (int i = lane; i < n; i += 32) a = fma(B[j * kSvdLd + i], B[j * kSvdLd + i], a);
         a = warp_sum_d(a);
         if (lane == 0) sig[j] = sqrt(a);
     }
@@ -159,7 +158,7 @@ jacobi_svd_kernel(int n, const T* __restrict__ R, int64_t ldr, T* __restrict__ U
     for (int e = tid; e < n * n; e += blockDim.x) {
         const int j = e / n, i = e % n, rk = rank[j];
         const double sj = sig[j];
-        U[(int64_t)rk * ldu + i] = (T)(sj > 0.0 ? B[j * n + i] / sj : 0.0);
+        U[(int64_t)rk * ldu + i] = (T)(sj > 0.0 ? B[j * kSvdLd + i] / sj : 0.0);
         if (want_v) V[(int64_t)rk * ldv + i] = (T)Vs[(size_t)j * np + i];
         if (i == 0) sigma[rk] = (T)sj;
     }
@@ -168,7 +167,7 @@ jacobi_svd_kernel(int n, const T* __restrict__ R, int64_t ldr, T* __restrict__ U
 template <typename T>
 inline size_t jacobi_svd_smem(int n) {
     const size_t np = (size_t)((n + 1) & ~1);
-    return sizeof(double) * (np * n + np * np + 2 * np) + sizeof(int) * np;
+    return sizeof(double) * (np * kSvdLd + np * np + 2 * np) + sizeof(int) * np;
 }
 
 // W(n x n) = U diag(max(sigma - tau, 0)) V^T; one block per column k of W.
