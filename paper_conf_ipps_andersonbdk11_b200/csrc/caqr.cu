@@ -994,7 +994,14 @@ static int svd_small_impl(int64_t n, const T* R, int64_t ldr, T* U, int64_t ldu,
             const char* e = getenv("CAQR_SVD_SWEEPS");  // diagnostics: cap the Jacobi sweeps
             return e ? std::max(1, atoi(e)) : 30;
         }();
-        jacobi_svd_kernel<T><<<1, kSvdThreads, smem, s>>>((int)n, R, ldr, U, ldu, sigma, V, ldv, tol, max_sweeps);
+        const char* be = getenv("CAQR_SVD_BLOCK");  // 0: always the single-CTA kernel
+        if (V == nullptr && n >= 32 && !(be && be[0] == '0')) {
+            // U, sigma only: block Jacobi over an 8-CTA cluster (DSMEM block moves)
+            jacobi_svd_block_kernel<T><<<kSvdCl, kSvdClT, 0, s>>>((int)n, R, ldr, U, ldu, sigma, tol, max_sweeps);
+        } else {
+            jacobi_svd_kernel<T><<<1, kSvdThreads, smem, s>>>((int)n, R, ldr, U, ldu, sigma, V, ldv, tol,
+                                                              max_sweeps);
+        }
         e = cudaGetLastError();
     }
     if (e != cudaSuccess) {
