@@ -300,9 +300,9 @@ jacobi_svd_block_kernel(int n, const T* __restrict__ R, int64_t ldr, T* __restri
                 const int dpos = pos == 0 ? 0 : (pos == 1 ? kSvdNBlk - 1 : pos - 1);
                 const int dcta = dpos < kSvdCl ? dpos : kSvdNBlk - 1 - dpos;
                 const int dslot = dpos < kSvdCl ? 0 : 1;
-                double* dst = cl.map_shared_rank(&buf[nxt][dslot * kSvdBlk][0], dcta);
-                const double* src = &buf[cur][slot * kSvdBlk][0];
-                for (int e = tid; e < kSvdBlk * kSvdLd; e += blockDim.x) dst[e] = src[e];
+                double2* dst = reinterpret_cast<double2*>(cl.map_shared_rank(&buf[nxt][dslot * kSvdBlk][0], dcta));
+                const double2* src = reinterpret_cast<const double2*>(&buf[cur][slot * kSvdBlk][0]);
+                for (int e = tid; e < kSvdBlk * kSvdLd / 2; e += blockDim.x) dst[e] = src[e];
                 int* dg = cl.map_shared_rank(&gidx[nxt][dslot * kSvdBlk], dcta);
                 if (tid < kSvdBlk) dg[tid] = gidx[cur][slot * kSvdBlk + tid];
             }
