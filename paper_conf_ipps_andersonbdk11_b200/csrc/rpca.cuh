@@ -198,7 +198,7 @@ jacobi_svd_block_kernel(int n, const T* __restrict__ R, int64_t ldr, T* __restri
     constexpr int NL = 2 * kSvdBlk;  // local columns: block A = 0..6, block B = 7..13
     __shared__ __align__(16) double buf[2][NL][kSvdLd];  // [cur/next][local column][row]
     __shared__ int gidx[2][NL];                             // global index of each local column
-    __shared__ double nrm[NL];
+    __shared__ double nrm2[2][NL];                          // squared column norms (travel with the blocks)
     __shared__ double sig0[kSvdNBlk * kSvdBlk];             // CTA 0: every sigma
     __shared__ int flag[2];                                 // CTA 0: "rotated in sweep s&1"
     __shared__ int s_rot;
@@ -222,7 +222,7 @@ jacobi_svd_block_kernel(int n, const T* __restrict__ R, int64_t ldr, T* __restri
             double a = 0.0;
             for (int i = lane; i < kSvdLd; i += 32) a = fma(buf[cur][lc][i], buf[cur][lc][i], a);
             a = warp_sum_d(a);
-            if (lane == 0) nrm[lc] = a;
+            if (lane == 0) nrm2[cur][lc] = a;
         }
     };
     // rotate local columns (p, q) so that they are orthogonal (half-warp hw)
@@ -249,7 +249,7 @@ jacobi_svd_block_kernel(int n, const T* __restrict__ R, int64_t ldr, T* __restri
         g += g1;
 #pragma unroll
         for (int o = 8; o > 0; o >>= 1) g += __shfl_xor_sync(hmask, g, o);
-        const double al = nrm[p], be = nrm[q];
+        const double al = nrm2[cur][p], be = nrm2[cur][q];
         __syncwarp(hmask);
         if (g * g > tol2 * (al * be) && g != 0.0) {
             const float df = (float)(be - al), gf = (float)g;
@@ -263,8 +263,8 @@ jacobi_svd_block_kernel(int n, const T* __restrict__ R, int64_t ldr, T* __restri
                 bq[16 * u] = sn * xp[u] + c * xq[u];
             }
             if (hl == 0) {
-                nrm[p] = al - t * g;
-                nrm[q] = be + t * g;
+                nrm2[cur][p] = al - t * g;
+                nrm2[cur][q] = be + t * g;
                 s_rot = 1;
             }
         }
@@ -283,10 +283,6 @@ jacobi_svd_block_kernel(int n, const T* __restrict__ R, int64_t ldr, T* __restri
         }
         for (int r = 0; r < kSvdNBlk - 1; ++r) {
             // ---- pairs across the two blocks held: 7 rounds of 7 disjoint pairs
-            if (r > 0) {
-                norms();
-                __syncthreads();
-            }
             for (int ir = 0; ir < kSvdBlk; ++ir) {
                 if (hw < kSvdBlk) rotate(hw, kSvdBlk + (hw + ir) % kSvdBlk);
                 __syncthreads();
@@ -305,6 +301,8 @@ jacobi_svd_block_kernel(int n, const T* __restrict__ R, int64_t ldr, T* __restri
                 for (int e = tid; e < kSvdBlk * kSvdLd / 2; e += blockDim.x) dst[e] = src[e];
                 int* dg = cl.map_shared_rank(&gidx[nxt][dslot * kSvdBlk], dcta);
                 if (tid < kSvdBlk) dg[tid] = gidx[cur][slot * kSvdBlk + tid];
+                double* dn = cl.map_shared_rank(&nrm2[nxt][dslot * kSvdBlk], dcta);
+                if (tid < kSvdBlk) dn[tid] = nrm2[cur][slot * kSvdBlk + tid];
             }
             cl.sync();
             cur = nxt;
