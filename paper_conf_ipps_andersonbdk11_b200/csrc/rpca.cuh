@@ -182,7 +182,7 @@ inline size_t jacobi_svd_smem(int n) {
 // distributed shared memory -- closed by one cluster barrier.  Every pair is
 // visited once per sweep, as in the single-CTA kernel, but in 7 + 15 x 7
 // cheap rounds on 8 SMs with 15 cluster barriers, instead of 99 rounds that
-// each carry all n/2 pairs on one SM (measured: 0.77 vs 1.58 ms at n = 100).
+// each carry all n/2 pairs on one SM (measured: 0.63 vs 1.58 ms at n = 100).
 constexpr int kSvdBlk = 7;     // columns per block
 constexpr int kSvdNBlk = 16;   // blocks (np <= 112)
 constexpr int kSvdCl = 8;      // CTAs per cluster (2 blocks each)
