@@ -773,8 +773,9 @@ __device__ __forceinline__ void apply_block(const Grp& G, const T* Vs, const T* 
     using V4 = typename Vec4<T>::type;
     constexpr int VN = Vec4<T>::n;
     const int tid = G.tid;
-    // W2 = op(T) W: thread (column c, rows jj = jg + 8q); T is zero below its
-    // diagonal, so full unrolled sums need no bounds.
+    // W2 = op(T) W: thread (column c, rows jj = 4 jg + q): the 4 T entries a
+    // thread needs per k are contiguous (one 16-byte load for Q^T); T is zero
+    // below its diagonal, so full unrolled sums need no bounds.
     T w2[4];
     {
         const int c = tid & 31, jg = tid >> 5;
@@ -785,27 +786,37 @@ __device__ __forceinline__ void apply_block(const Grp& G, const T* Vs, const T* 
             T wc[16];
 #pragma unroll
             for (int k = 0; k < 16; ++k) wc[k] = W[(h + k) * kTS + c];
+            if (trans) {
 #pragma unroll
-            for (int q = 0; q < 4; ++q) {
-                const int jj = jg + 8 * q;
-                T a0 = 0, a1 = 0;
+                for (int k = 0; k < 16; ++k) {
+                    T tq[4];
 #pragma unroll
-                for (int k = 0; k < 16; k += 2) {
-                    if (trans) {
-                        a0 = fma(Tt[(h + k) * kTS + jj], wc[k], a0);
-                        a1 = fma(Tt[(h + k + 1) * kTS + jj], wc[k + 1], a1);
-                    } else {
+                    for (int hh = 0; hh < 4 / VN; ++hh) {
+                        const V4 t4 = *reinterpret_cast<const V4*>(Tt + (h + k) * kTS + 4 * jg + hh * VN);
+#pragma unroll
+                        for (int e = 0; e < VN; ++e) tq[hh * VN + e] = vget<T>(t4, e);
+                    }
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) w2[q] = fma(tq[q], wc[k], w2[q]);
+                }
+            } else {
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int jj = 4 * jg + q;
+                    T a0 = 0, a1 = 0;
+#pragma unroll
+                    for (int k = 0; k < 16; k += 2) {
                         a0 = fma(Tt[jj * kTS + h + k], wc[k], a0);
                         a1 = fma(Tt[jj * kTS + h + k + 1], wc[k + 1], a1);
                     }
+                    w2[q] += a0 + a1;
                 }
-                w2[q] += a0 + a1;
             }
         }
     }
     gsync(G);
 #pragma unroll
-    for (int q = 0; q < 4; ++q) W[((tid >> 5) + 8 * q) * kTS + (tid & 31)] = w2[q];
+    for (int q = 0; q < 4; ++q) W[(4 * (tid >> 5) + q) * kTS + (tid & 31)] = w2[q];
     gsync(G);
     if constexpr (sizeof(T) == 4) {
         gemm2_mma<true>(G, Vs, const_cast<T*>(Cs), W, RGP, R32);
