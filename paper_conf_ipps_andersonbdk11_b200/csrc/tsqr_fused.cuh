@@ -766,10 +766,31 @@ __device__ __forceinline__ void gemm2_mma(const Grp& G, const float* Vs, float* 
     }
 }
 
+// This thread's two row quads r = 4 (lane + 32 b), b < 2, of a node's gathered
+// rows (<= 256): absolute row offset and the number of rows < RG in the quad.
+// Fixed per (node, panel), so the 16-byte staging and write-back of every
+// trailing block reuse them instead of re-deriving them element by element.
+struct RowQuads {
+    int64_t off[2];
+    int cnt[2];
+};
+__device__ __forceinline__ RowQuads row_quads(const NodeRows& nr, int RG) {
+    const int lane = threadIdx.x & 31;
+    RowQuads q;
+#pragma unroll
+    for (int b = 0; b < 2; ++b) {
+        const int r = 4 * (lane + 32 * b);
+        q.cnt[b] = max(0, min(4, RG - r));
+        q.off[b] = q.cnt[b] > 0 ? gathered_row(nr, r) : 0;
+    }
+    return q;
+}
+
 template <typename T>
 __device__ __forceinline__ void apply_block(const Grp& G, const T* Vs, const T* Cs, const T* Tt, T* W, int RGP, int R32,
                                             int RG, int wp, int trans, const NodeRows& nr, T* C,
-                                            int64_t ldc, int64_t cb0, int ncb, bool vec = false) {
+                                            int64_t ldc, int64_t cb0, int ncb, bool vec = false,
+                                            const RowQuads* rq = nullptr) {
     using V4 = typename Vec4<T>::type;
     constexpr int VN = Vec4<T>::n;
     const int tid = G.tid;
@@ -874,7 +895,21 @@ __device__ __forceinline__ void apply_block(const Grp& G, const T* Vs, const T* 
     gsync(G);
     {
         const int warp = tid >> 5, lane = tid & 31;
-        if (sizeof(T) == 4 && vec) {  // float4 stores: rows 4q..4q+3 lie in one segment
+        if (sizeof(T) == 4 && vec && rq) {  // float4 stores, precomputed row quads
+            for (int c = warp; c < ncb; c += kWarps) {
+                T* ccol = C + (cb0 + c) * ldc;
+                const T* cs = Cs + (size_t)c * RGP;
+#pragma unroll
+                for (int u = 0; u < 2; ++u) {
+                    const int r = 4 * (lane + 32 * u);
+                    if (rq->cnt[u] == 4) {
+                        *reinterpret_cast<float4*>(ccol + rq->off[u]) = *reinterpret_cast<const float4*>(cs + r);
+                    } else {
+                        for (int q = 0; q < rq->cnt[u]; ++q) ccol[rq->off[u] + q] = cs[r + q];
+                    }
+                }
+            }
+        } else if (sizeof(T) == 4 && vec) {  // float4 stores: rows 4q..4q+3 lie in one segment
             for (int c = warp; c < ncb; c += kWarps) {
                 T* ccol = C + (cb0 + c) * ldc;
                 const T* cs = Cs + (size_t)c * RGP;
@@ -905,9 +940,27 @@ __device__ __forceinline__ void apply_block(const Grp& G, const T* Vs, const T* 
 // aligned, lda % 4 == 0, row segments starting on multiples of 4).  Caller
 // waits (cp.async.wait_group) and synchronises.
 __device__ __forceinline__ void stage_cols_cp(const Grp& G, float* S, int RGP, int R32, const float* M, int64_t ld,
-                                              int64_t col0, int ncol, const NodeRows& nr, int RG, bool vec) {
+                                              int64_t col0, int ncol, const NodeRows& nr, int RG, bool vec,
+                                              const RowQuads* rq = nullptr) {
     const int warp = G.tid >> 5, lane = G.tid & 31;
-    if (vec) {
+    if (vec && rq) {
+#pragma unroll
+        for (int a = 0; a < 4; ++a) {
+            const int jj = warp + 8 * a;
+            const float* mc = M + (col0 + min(jj, max(ncol - 1, 0))) * ld;
+#pragma unroll
+            for (int b = 0; b < 2; ++b) {
+                const int r = 4 * (lane + 32 * b);
+                if (r < R32) {
+                    const int valid = jj < ncol ? rq->cnt[b] : 0;
+                    const unsigned dst = (unsigned)__cvta_generic_to_shared(S + (size_t)jj * RGP + r);
+                    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(mc + rq->off[b]),
+                                 "r"(valid * 4)
+                                 : "memory");
+                }
+            }
+        }
+    } else if (vec) {
 #pragma unroll
         for (int a = 0; a < 4; ++a) {
             const int jj = warp + 8 * a;
@@ -1148,12 +1201,13 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
             // panel can be staged from Cs)
             const int64_t tfirst = c0 + 32, tend = g.col0 + g.ncols;
             const int nblk = tend > tfirst ? (int)((tend - tfirst + 31) / 32) : 0;
+            const bool vec_p = vec && (nr.n0 % 4 == 0);
+            const RowQuads rq = row_quads(nr, RG);
             for (int ib = 0; ib < nblk; ++ib) {
                 const int64_t cb0 = tfirst + 32 * ((ib + 1) % nblk);
                 const int ncb = (int)(tend - cb0 < 32 ? tend - cb0 : 32);
-                const bool vec_p = vec && (nr.n0 % 4 == 0);
                 if constexpr (sizeof(T) == 4) {
-                    stage_cols_cp(G0, Cs, RGP, R32, A, g.lda, cb0, ncb, nr, RG, vec_p);
+                    stage_cols_cp(G0, Cs, RGP, R32, A, g.lda, cb0, ncb, nr, RG, vec_p, &rq);
                     asm volatile("cp.async.wait_group 0;" ::: "memory");
                 } else {
                     stage_cols(G0, Cs, RGP, R32, static_cast<const T*>(A), g.lda, cb0, ncb, nr, RG, false, p);
@@ -1165,7 +1219,7 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
                 else
                     gemm_vtc(G0, P, Cs, RGP, R32, Wp, W);
                 CAQR_PROF(7);
-                apply_block(G0, P, Cs, Tt, W, RGP, R32, RG, wp, 1, nr, A, g.lda, cb0, ncb, vec_p);
+                apply_block(G0, P, Cs, Tt, W, RGP, R32, RG, wp, 1, nr, A, g.lda, cb0, ncb, vec_p, &rq);
                 CAQR_PROF(8);
             }
             // ---- publish ----------------------------------------------------------
