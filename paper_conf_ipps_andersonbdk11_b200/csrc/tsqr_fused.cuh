@@ -790,7 +790,7 @@ template <typename T>
 __device__ __forceinline__ void apply_block(const Grp& G, const T* Vs, const T* Cs, const T* Tt, T* W, int RGP, int R32,
                                             int RG, int wp, int trans, const NodeRows& nr, T* C,
                                             int64_t ldc, int64_t cb0, int ncb, bool vec = false,
-                                            const RowQuads* rq = nullptr) {
+                                            const RowQuads* rq = nullptr, T* W2buf = nullptr) {
     using V4 = typename Vec4<T>::type;
     constexpr int VN = Vec4<T>::n;
     const int tid = G.tid;
@@ -835,12 +835,15 @@ __device__ __forceinline__ void apply_block(const Grp& G, const T* Vs, const T* 
             }
         }
     }
-    gsync(G);
+    // W2 into a separate buffer when given (no barrier between reading W and
+    // writing W2), else over W
+    T* W2 = W2buf ? W2buf : W;
+    if (!W2buf) gsync(G);
 #pragma unroll
-    for (int q = 0; q < 4; ++q) W[(4 * (tid >> 5) + q) * kTS + (tid & 31)] = w2[q];
+    for (int q = 0; q < 4; ++q) W2[(4 * (tid >> 5) + q) * kTS + (tid & 31)] = w2[q];
     gsync(G);
     if constexpr (sizeof(T) == 4) {
-        gemm2_mma<true>(G, Vs, const_cast<T*>(Cs), W, RGP, R32);
+        gemm2_mma<true>(G, Vs, const_cast<T*>(Cs), W2, RGP, R32);
     } else {
     const int nq = R32 / 4;
     for (int u = tid; u < nq * 4; u += kThreads) {
@@ -868,7 +871,7 @@ __device__ __forceinline__ void apply_block(const Grp& G, const T* Vs, const T* 
             T wv[8];
 #pragma unroll
             for (int h = 0; h < 8 / VN; ++h) {
-                const V4 t4 = *reinterpret_cast<const V4*>(W + jj * kTS + cbase + h * VN);
+                const V4 t4 = *reinterpret_cast<const V4*>(W2 + jj * kTS + cbase + h * VN);
 #pragma unroll
                 for (int k = 0; k < VN; ++k) wv[h * VN + k] = vget<T>(t4, k);
             }
@@ -1219,7 +1222,7 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
                 else
                     gemm_vtc(G0, P, Cs, RGP, R32, Wp, W);
                 CAQR_PROF(7);
-                apply_block(G0, P, Cs, Tt, W, RGP, R32, RG, wp, 1, nr, A, g.lda, cb0, ncb, vec_p, &rq);
+                apply_block(G0, P, Cs, Tt, W, RGP, R32, RG, wp, 1, nr, A, g.lda, cb0, ncb, vec_p, &rq, Wp);
                 CAQR_PROF(8);
             }
             // ---- publish ----------------------------------------------------------
