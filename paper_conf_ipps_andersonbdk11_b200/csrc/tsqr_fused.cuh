@@ -484,7 +484,11 @@ __device__ __forceinline__ void factor_panel_wb4(const Grp& G, T* P, int RGP, in
             }
             T tt[16];
 #pragma unroll
-            for (int k = 0; k < 16; ++k) tt[k] = Tb[b * 16 + k];
+            for (int k = 0; k < 16; k += Vec4<T>::n) {
+                const typename Vec4<T>::type t4 = *reinterpret_cast<const typename Vec4<T>::type*>(Tb + b * 16 + k);
+#pragma unroll
+                for (int e = 0; e < Vec4<T>::n; ++e) tt[k + e] = vget<T>(t4, e);
+            }
 #pragma unroll
             for (int q = 0; q < 4; ++q) {
                 T w2[4];
@@ -1152,17 +1156,41 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
                                   ? ldcg(A + (c0 + jj) * g.lda + gathered_row(nr, lane))
                                   : T(0);
                 }
+                if (sizeof(T) == 4 && (leaf || nr.n0 == 32)) {
+                    // 16-byte copies: a leaf's rows r come from Cs row r + 32, a chain
+                    // step's rows r >= 32 from Cs row r (rows < 32: the slot's heads)
 #pragma unroll
-                for (int a = 0; a < 4; ++a) {
-                    const int jj = warp + 8 * a;
-                    T* pc = P + (size_t)jj * RGP;
-                    const T* cc = Cs + (size_t)jj * RGP;
-                    for (int r = lane; r < R32; r += 32) {
-                        T v;
-                        if (leaf) v = (r < RG && jj < wp) ? cc[padr<T>(r + 32)] : T(0);
-                        else if (r < nr.n0) v = head[a];
-                        else v = (r < RG && jj < wp) ? cc[padr<T>(r - nr.n0 + 32)] : T(0);
-                        pc[padr<T>(r)] = v;
+                    for (int a = 0; a < 4; ++a) {
+                        const int jj = warp + 8 * a;
+                        float* pc = reinterpret_cast<float*>(P) + (size_t)jj * RGP;
+                        const float* cc = reinterpret_cast<const float*>(Cs) + (size_t)jj * RGP;
+                        if (!leaf) pc[lane] = head[a];
+#pragma unroll
+                        for (int u = 0; u < 2; ++u) {
+                            const int r4 = 4 * (lane + 32 * u);
+                            if (r4 >= R32 || (!leaf && r4 < 32)) continue;
+                            float4 v = *reinterpret_cast<const float4*>(cc + r4 + (leaf ? 32 : 0));
+                            const bool ok = jj < wp;
+                            v.x = ok && r4 < RG ? v.x : 0.f;
+                            v.y = ok && r4 + 1 < RG ? v.y : 0.f;
+                            v.z = ok && r4 + 2 < RG ? v.z : 0.f;
+                            v.w = ok && r4 + 3 < RG ? v.w : 0.f;
+                            *reinterpret_cast<float4*>(pc + r4) = v;
+                        }
+                    }
+                } else {
+#pragma unroll
+                    for (int a = 0; a < 4; ++a) {
+                        const int jj = warp + 8 * a;
+                        T* pc = P + (size_t)jj * RGP;
+                        const T* cc = Cs + (size_t)jj * RGP;
+                        for (int r = lane; r < R32; r += 32) {
+                            T v;
+                            if (leaf) v = (r < RG && jj < wp) ? cc[padr<T>(r + 32)] : T(0);
+                            else if (r < nr.n0) v = head[a];
+                            else v = (r < RG && jj < wp) ? cc[padr<T>(r - nr.n0 + 32)] : T(0);
+                            pc[padr<T>(r)] = v;
+                        }
                     }
                 }
             } else {
