@@ -590,7 +590,8 @@ __device__ __forceinline__ void gemm_vtc(const Grp& G, const T* Vs, const T* Cs,
 // T[0:j,j] = -tau_j T[0:j,0:j] G[0:j,j].  One warp; lane i keeps row i of T in
 // registers; 4 independent accumulation chains.
 template <typename T>
-__device__ __forceinline__ void build_t(const Grp& Gr, const T* G, const T* tau_s, int wp, T* Tt) {
+__device__ __forceinline__ void build_t(const Grp& Gr, const T* G, const T* tau_s, int wp, T* Tt,
+                                       T* tglobal = nullptr) {
     const int lane = Gr.tid & 31;
     if (Gr.tid >= 32) return;
     T row[32];
@@ -611,6 +612,9 @@ __device__ __forceinline__ void build_t(const Grp& Gr, const T* G, const T* tau_
     }
 #pragma unroll
     for (int j = 0; j < 32; ++j) Tt[lane * kTS + j] = row[j];
+    if (tglobal)  // the workspace's column-major T block: coalesced across lanes
+#pragma unroll
+        for (int j = 0; j < 32; ++j) tglobal[j * 32 + lane] = row[j];
 }
 
 // C(RG x 32, in Cs) <- C - V (op(T) W) ; written straight to global rows.
@@ -1203,15 +1207,8 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
             CAQR_PROF(3);
             CAQR_PROF(4);
             gemm_vtc(G0, P, P, RGP, R32, Wp, W);  // G = V^T V
-            build_t(G0, W, tau_s, wp, Tt);
+            build_t(G0, W, tau_s, wp, Tt, Tws + nr.tblk * (kPW * kPW));
             __syncthreads();
-            {
-                T* tb = Tws + nr.tblk * (kPW * kPW);
-                for (int e = threadIdx.x; e < kPW * kPW; e += kThreads) {
-                    const int r = e & 31, c = e >> 5;
-                    tb[e] = Tt[r * kTS + c];
-                }
-            }
             // wait for the children's trailing updates before touching later
             // columns, then publish "factored" (the stored R / V of panel p are in A)
             __threadfence();
