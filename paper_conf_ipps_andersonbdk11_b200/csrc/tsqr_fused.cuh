@@ -515,15 +515,37 @@ __device__ __forceinline__ void factor_panel_wb4(const Grp& G, T* P, int RGP, in
         // masks) to global, the V form (unit head, zeros elsewhere) into P,
         // zero columns beyond wp -- no extra pass over P
         const NodeRows& nr = *out_nr;
+        // per row (shared by the 4 columns): segment, absolute row, and the
+        // structure test's row key -- r for segment 0 (stored iff r <= jj when
+        // it is an R slot), r - n0 - 32p for an upper-triangular segment 1
+        // (stored iff key <= jj), -inf-like for a dense one
+        int64_t grow[8];
+        int key[8];
+        bool seg0[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            const int r = lane + 32 * i;
+            seg0[i] = r < nr.n0;
+            grow[i] = seg0[i] ? nr.r0 + r : nr.r1 + (r - nr.n0);
+            key[i] = seg0[i] ? (nr.seg0_tri ? r : -1) : (nr.seg1_upper ? r - nr.n0 - 32 * out_p : -1);
+        }
 #pragma unroll
         for (int q = 0; q < 4; ++q) {
-            T* col = out_A + (out_c0 + cb + q) * out_lda;
+            const int jj = cb + q;
+            T* col = out_A + (out_c0 + jj) * out_lda;
+            T* pcol = P + (size_t)jj * RGP;
 #pragma unroll
             for (int i = 0; i < 8; ++i) {
                 const int r = lane + 32 * i;
                 const bool in = q < nc && r < RG;
-                if (in && panel_entry_stored(nr, r, cb + q, out_p)) col[gathered_row(nr, r)] = x[q][i];
-                P[(size_t)(cb + q) * RGP + padr<T>(r)] = in ? v_entry<T>(nr, r, cb + q, out_p, x[q][i]) : T(0);
+                const bool stored = key[i] <= jj;
+                if (in && stored) col[grow[i]] = x[q][i];
+                T v = T(0);
+                if (in) {
+                    if (seg0[i]) v = nr.seg0_tri ? (r == jj ? T(1) : T(0)) : (r > jj ? x[q][i] : (r == jj ? T(1) : T(0)));
+                    else v = stored ? x[q][i] : T(0);
+                }
+                pcol[padr<T>(r)] = v;
             }
         }
     } else {
