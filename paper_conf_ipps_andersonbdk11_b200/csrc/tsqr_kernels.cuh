@@ -493,7 +493,8 @@ __device__ __forceinline__ void update_node(const Geom& g, const T* A, const T* 
     __syncthreads();
     }
     // ---- W2 = T^T W (Q^T) or T W (Q); T upper triangular (Tt[r][c] = T[r][c])
-    // thread (column c, rows jj = jg + 8q); unrolled, T's zeros need no bounds
+    // thread (column c, rows jj = 4 jg + q): its 4 T entries per k are one
+    // 16-byte load (Q^T); unrolled, T's zeros need no bounds
     T w2[4];
     {
         const int c = tid & 31, jg = tid >> 5;
@@ -504,23 +505,34 @@ __device__ __forceinline__ void update_node(const Geom& g, const T* A, const T* 
             T wc[8];
 #pragma unroll
             for (int k2 = 0; k2 < 8; ++k2) wc[k2] = W[(h + k2) * kTS + c];
+            if (trans) {
 #pragma unroll
-            for (int q = 0; q < 4; ++q) {
-                const int jj = jg + 8 * q;
-                T acc = T(0);
+                for (int k2 = 0; k2 < 8; ++k2) {
+                    T tq[4];
 #pragma unroll
-                for (int k2 = 0; k2 < 8; ++k2)
-                    acc = fma(trans ? Tt[(h + k2) * kTS + jj] : Tt[jj * kTS + h + k2], wc[k2], acc);
-                w2[q] += acc;
+                    for (int hh = 0; hh < 4 / VN; ++hh) {
+                        const V4 t4 = *reinterpret_cast<const V4*>(Tt + (h + k2) * kTS + 4 * jg + hh * VN);
+#pragma unroll
+                        for (int e = 0; e < VN; ++e) tq[hh * VN + e] = vget<T>(t4, e);
+                    }
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) w2[q] = fma(tq[q], wc[k2], w2[q]);
+                }
+            } else {
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int jj = 4 * jg + q;
+                    T acc = T(0);
+#pragma unroll
+                    for (int k2 = 0; k2 < 8; ++k2) acc = fma(Tt[jj * kTS + h + k2], wc[k2], acc);
+                    w2[q] += acc;
+                }
             }
         }
     }
     __syncthreads();
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
-        const int e = tid + q * kThreads;
-        W[(e >> 5) * kTS + (e & 31)] = w2[q];
-    }
+    for (int q = 0; q < 4; ++q) W[(4 * (tid >> 5) + q) * kTS + (tid & 31)] = w2[q];
     __syncthreads();
 
     if constexpr (MMA) {
@@ -529,7 +541,17 @@ __device__ __forceinline__ void update_node(const Geom& g, const T* A, const T* 
         for (int c = warp; c < ncb; c += kWarps) {
             T* ccol = C + (cb0 + c) * ldc;
             const T* cs = Cs + (size_t)c * RGP;
-            for (int r = lane; r < RG; r += 32) ccol[gathered_row(nr, r)] = cs[r];
+            if (vec_p) {  // rows 4q..4q+3: one segment, 16-byte aligned
+                for (int r = 4 * lane; r < RG; r += 128) {
+                    if (r + 4 <= RG)
+                        *reinterpret_cast<float4*>(reinterpret_cast<float*>(ccol) + gathered_row(nr, r)) =
+                            *reinterpret_cast<const float4*>(reinterpret_cast<const float*>(cs) + r);
+                    else
+                        for (int q = r; q < RG; ++q) ccol[gathered_row(nr, q)] = cs[q];
+                }
+            } else {
+                for (int r = lane; r < RG; r += 32) ccol[gathered_row(nr, r)] = cs[r];
+            }
         }
     } else {
     // ---- C -= V W2 : thread = (4 consecutive rows, 8 consecutive columns) ---
