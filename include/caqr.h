@@ -156,6 +156,46 @@ int caqr_combine_apply_f32(int P, int64_t n, const float *Rstack, int64_t ld, co
 int caqr_combine_apply_f64(int P, int64_t n, const double *Rstack, int64_t ld, const void *ws,
                            int trans, int64_t k, double *C, int64_t ldc, caqr_stream_t stream);
 
+/* ---- Host-streamed factorisation (end-to-end from host memory) ------------
+ * A = QR of a matrix that lives in HOST memory (pinned for overlap).  The rows
+ * are split into `chunks` row blocks, chunk c = rows [m*c/chunks,
+ * m*(c+1)/chunks); each block's H2D copy runs on a copy engine (a library copy
+ * stream) while the previous blocks are factored on `stream` by caqr_factor_*;
+ * the chunks' R factors are then reduced by caqr_combine_* — the extra tree
+ * level of the distributed TSQR the paper cites, here with row
+ * blocks of one GPU as its leaves.  Not in the paper (its runtimes exclude the
+ * transfer); it hides the PCIe copy behind the factorisation.
+ *   m, n        m >= n >= 0                                       (info -1, -2)
+ *   chunks      1..1024; if > 1: n <= 256 and m/chunks >= n       (info -3)
+ *   A_host      host, m x n column-major, lda_host >= max(1,m)    (info -4, -5)
+ *   A           device, m x n, lda >= max(1,m): receives A, then   (info -6, -7)
+ *               each chunk's implicit-Q representation (as caqr_factor_* on
+ *               the chunk's rows)
+ *   R           device, n x n, ldr >= n: the global R, strict      (info -8, -9)
+ *               lower zeroed
+ *   ws          device, ws_bytes >= caqr_factor_host_workspace_bytes (-10, -11)
+ *   opts        plan of every chunk's factorisation (NULL = default) (-12)
+ * Q = diag(Q_0..Q_{S-1}) * [rows n of each chunk -> Qc], Qc the combine's
+ * orthogonal factor.  caqr_factor_host_layout(..., c, out3) gives, for
+ * c < chunks, out3 = {first row, rows, byte offset of the chunk's workspace in
+ * ws}; for c = chunks, {0, chunks*n, offset of the R stack ((chunks*n) x n,
+ * ld chunks*n: the combine's tree vectors)}; for c = chunks+1, {0, 0, offset
+ * of the combine workspace}: with them, caqr_apply_qt_* per chunk followed by
+ * caqr_combine_apply_* on the chunks' top n rows applies Q^T (as for the
+ * row-sharded multi-GPU factorization).  The caller keeps A_host unchanged
+ * until the stream reaches the end of the call.  Layout query: 0, or -3 (bad
+ * m, n, chunks, dtype, opts), -6 (c out of range), -7 (out3 NULL).
+ * caqr_factor_host_workspace_bytes returns 0 on illegal arguments. */
+size_t caqr_factor_host_workspace_bytes(int64_t m, int64_t n, int chunks, int dtype, const caqr_opts *opts);
+int caqr_factor_host_layout(int64_t m, int64_t n, int chunks, int dtype, const caqr_opts *opts, int c,
+                            int64_t *out3);
+int caqr_factor_host_f32(int64_t m, int64_t n, int chunks, const float *A_host, int64_t lda_host, float *A,
+                         int64_t lda, float *R, int64_t ldr, void *ws, size_t ws_bytes,
+                         const caqr_opts *opts, caqr_stream_t stream);
+int caqr_factor_host_f64(int64_t m, int64_t n, int chunks, const double *A_host, int64_t lda_host, double *A,
+                         int64_t lda, double *R, int64_t ldr, void *ws, size_t ws_bytes,
+                         const caqr_opts *opts, caqr_stream_t stream);
+
 /* Q (m x n, ldq >= m) = [I_n; 0]: the start of an explicit Q (caqr_form_q does
  * it internally); used with caqr_combine_apply / caqr_apply_q to form the rows
  * of a row-sharded factorization's Q on each rank.

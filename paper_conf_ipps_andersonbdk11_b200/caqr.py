@@ -76,6 +76,14 @@ def lib() -> ctypes.CDLL:
             f = getattr(L, f"caqr_dist_factor_{suf}")
             f.argtypes = [vp, i64, i64, vp, i64, vp, i64, vp, sz, vp, vp, sz, op, vp]
             f.restype = ip
+        for suf in ("f32", "f64"):
+            f = getattr(L, f"caqr_factor_host_{suf}")
+            f.argtypes = [i64, i64, ip, vp, i64, vp, i64, vp, i64, vp, sz, op, vp]
+            f.restype = ip
+        L.caqr_factor_host_workspace_bytes.argtypes = [i64, i64, ip, ip, op]
+        L.caqr_factor_host_workspace_bytes.restype = sz
+        L.caqr_factor_host_layout.argtypes = [i64, i64, ip, ip, op, ip, ctypes.POINTER(ctypes.c_int64)]
+        L.caqr_factor_host_layout.restype = ip
         L.caqr_combine_workspace_bytes.argtypes = [ip, i64, ip]
         L.caqr_combine_workspace_bytes.restype = sz
         L.caqr_strerror.argtypes = [ip]
@@ -167,8 +175,8 @@ def _dtype_code(t) -> Tuple[int, str]:
     raise TypeError(f"caqr: dtype {t.dtype} not supported (float32 / float64)")
 
 
-def _colmajor(t, name: str):
-    if not t.is_cuda:
+def _colmajor(t, name: str, host: bool = False):
+    if not host and not t.is_cuda:
         raise ValueError(f"caqr: {name} must be a CUDA tensor (no CPU path)")
     if t.dim() != 2:
         raise ValueError(f"caqr: {name} must be 2-D")
@@ -229,6 +237,45 @@ def caqr_factor(A, R=None, ws=None, opts: Optional[Opts] = None, stream=None):
                                                  _optp(opts), _stream(stream))
     _check(f"caqr_factor_{suf}", info)
     return R, ws
+
+
+def caqr_factor_host_workspace_bytes(m: int, n: int, chunks: int, dtype: int = CAQR_F32,
+                                     opts: Optional[Opts] = None) -> int:
+    return int(lib().caqr_factor_host_workspace_bytes(m, n, chunks, dtype, _optp(opts)))
+
+
+def caqr_factor_host_layout(m: int, n: int, chunks: int, c: int, dtype: int = CAQR_F32,
+                            opts: Optional[Opts] = None) -> Tuple[int, int, int]:
+    out = (ctypes.c_int64 * 3)()
+    _check("caqr_factor_host_layout", lib().caqr_factor_host_layout(m, n, chunks, dtype, _optp(opts), c, out))
+    return int(out[0]), int(out[1]), int(out[2])
+
+
+def caqr_factor_host(A_host, chunks: int, A=None, R=None, ws=None, opts: Optional[Opts] = None, stream=None):
+    """Factor a column-major HOST matrix (pinned for overlap): chunked H2D copies
+    overlapped with the chunks' factorisations, then the combine.  Returns
+    (A, R, ws) on the device (A/ws: the chunked implicit Q, see caqr.h)."""
+    torch = _torch()
+    if A_host.is_cuda:
+        raise ValueError("A_host must be a host tensor")
+    code, suf = _dtype_code(A_host)
+    m, n = A_host.shape
+    ph, ldh = _colmajor(A_host, "A_host", host=True)
+    if A is None:
+        A = colmajor_empty(m, n, A_host.dtype, "cuda")
+    pa, lda = _colmajor(A, "A")
+    if R is None:
+        R = colmajor_empty(n, n, A_host.dtype, A.device)
+    pr, ldr = _colmajor(R, "R")
+    need = caqr_factor_host_workspace_bytes(m, n, chunks, code, opts)
+    if need == 0 and n > 0:
+        raise CaqrError("caqr_factor_host_workspace_bytes", -3, "illegal size/chunks/opts")
+    if ws is None:
+        ws = torch.empty(max(need, 1), dtype=torch.uint8, device=A.device)
+    info = getattr(lib(), f"caqr_factor_host_{suf}")(m, n, chunks, ph, ldh, pa, lda, pr, ldr, ws.data_ptr(),
+                                                      ws.numel(), _optp(opts), _stream(stream))
+    _check(f"caqr_factor_host_{suf}", info)
+    return A, R, ws
 
 
 def _apply(name, A, ws, C, n, opts, stream):

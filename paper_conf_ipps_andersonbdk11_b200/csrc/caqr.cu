@@ -1061,6 +1061,116 @@ static int set_identity_impl(int64_t m, int64_t n, T* Q, int64_t ldq, cudaStream
     set_identity_kernel<T><<<grid, 256, 0, s>>>(m, n, Q, ldq);
     return launch_status();
 }
+// ---- Host-streamed factorisation (caqr_factor_host_*) ----------------------
+// The row chunks of A are a one-GPU instance of the distributed TSQR the paper
+// cites: chunk c is factored by the ordinary path as soon as its
+// H2D copy (a copy engine, second stream) has landed, while later chunks are
+// still in flight; the chunks' R factors are then combined by the structured
+// tree of caqr_combine.  Chunk c = rows [m*c/S, m*(c+1)/S).
+static inline int64_t host_chunk_row(int64_t m, int S, int c) { return (int64_t)(((__int128)m * c) / S); }
+static inline size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
+
+// Offsets of the chunk workspaces, the R stack and the combine workspace.
+// Returns 0 on illegal arguments.
+static size_t host_layout(int64_t m, int64_t n, int S, int dtype, const caqr_opts* opts, int c,
+                          int64_t* row0, int64_t* rows, size_t* off) {
+    if (m < 0 || n < 0 || n > m || S < 1 || S > 1024 || (dtype != CAQR_F32 && dtype != CAQR_F64)) return 0;
+    if (S > 1 && (n > kMaxGroup || m / S < n)) return 0;
+    const size_t es = dtype == CAQR_F64 ? 8 : 4;
+    size_t o = 0;
+    for (int q = 0; q < S; ++q) {
+        const int64_t r0 = host_chunk_row(m, S, q), mc = host_chunk_row(m, S, q + 1) - r0;
+        const size_t wb = caqr_workspace_bytes(mc, n, dtype, opts);
+        if (wb == 0) return 0;
+        if (q == c) {
+            *row0 = r0;
+            *rows = mc;
+            *off = o;
+        }
+        o += align256(wb);
+    }
+    const size_t rstack = align256((size_t)S * n * n * es);
+    if (c == S) { *row0 = 0; *rows = (int64_t)S * n; *off = o; }           // the R stack
+    o += rstack;
+    const size_t cw = S > 1 ? caqr_combine_workspace_bytes(S, n, dtype) : 256;
+    if (cw == 0) return 0;
+    if (c == S + 1) { *row0 = 0; *rows = 0; *off = o; }                    // the combine workspace
+    return o + align256(cw);
+}
+
+// One copy stream and a pool of events per device for the H2D pipeline.
+static bool copy_stream(cudaStream_t* cs, cudaEvent_t** evs) {
+    static std::mutex mu;
+    static cudaStream_t streams[64] = {};
+    static cudaEvent_t pool[64][1025] = {};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev >= 64) return false;
+    std::lock_guard<std::mutex> lk(mu);
+    if (!streams[dev]) {
+        if (cudaStreamCreateWithFlags(&streams[dev], cudaStreamNonBlocking) != cudaSuccess) return false;
+        for (int i = 0; i < 1025; ++i)
+            if (cudaEventCreateWithFlags(&pool[dev][i], cudaEventDisableTiming) != cudaSuccess) return false;
+    }
+    *cs = streams[dev];
+    *evs = pool[dev];
+    return true;
+}
+
+template <typename T>
+static int factor_host_impl(int64_t m, int64_t n, int S, const T* Ah, int64_t ldh, T* A, int64_t lda, T* R,
+                            int64_t ldr, void* ws, size_t ws_bytes, const caqr_opts* opts, cudaStream_t s,
+                            int dtype) {
+    if (m < 0) return -1;
+    if (n < 0 || n > m) return -2;
+    if (S < 1 || S > 1024 || (S > 1 && (n > kMaxGroup || m / S < n))) return -3;
+    if (ldh < std::max<int64_t>(1, m)) return -5;
+    if (lda < std::max<int64_t>(1, m)) return -7;
+    if (ldr < std::max<int64_t>(1, n)) return -9;
+    int64_t r0, mc;
+    size_t off;
+    const size_t need = host_layout(m, n, S, dtype, opts, 0, &r0, &mc, &off);
+    if (need == 0) return -12;
+    if (m == 0 || n == 0) return 0;
+    if (!Ah) return -4;
+    if (!A) return -6;
+    if (!R) return -8;
+    if (!ws) return -10;
+    if (ws_bytes < need) return -11;
+    cudaStream_t cs;
+    cudaEvent_t* ev;
+    if (!copy_stream(&cs, &ev)) return CAQR_ERR_CUDA;
+    // The copies may overwrite A only after the work already queued on s.
+    if (cudaEventRecord(ev[S], s) != cudaSuccess || cudaStreamWaitEvent(cs, ev[S], 0) != cudaSuccess)
+        return CAQR_ERR_CUDA;
+    char* wsb = static_cast<char*>(ws);
+    for (int c = 0; c < S; ++c) {
+        host_layout(m, n, S, dtype, opts, c, &r0, &mc, &off);
+        if (cudaMemcpy2DAsync(A + r0, lda * sizeof(T), Ah + r0, ldh * sizeof(T), mc * sizeof(T), n,
+                              cudaMemcpyHostToDevice, cs) != cudaSuccess ||
+            cudaEventRecord(ev[c], cs) != cudaSuccess) {
+            g_last_cuda_error = (int)cudaGetLastError();
+            return CAQR_ERR_CUDA;
+        }
+    }
+    int64_t rs0, rsn;
+    size_t rs_off, cw_off;
+    host_layout(m, n, S, dtype, opts, S, &rs0, &rsn, &rs_off);
+    host_layout(m, n, S, dtype, opts, S + 1, &rs0, &rsn, &cw_off);
+    T* Rs = reinterpret_cast<T*>(wsb + rs_off);
+    const int64_t ld = (int64_t)S * n;
+    int rc = 0;
+    for (int c = 0; c < S && !rc; ++c) {
+        host_layout(m, n, S, dtype, opts, c, &r0, &mc, &off);
+        if (cudaStreamWaitEvent(s, ev[c], 0) != cudaSuccess) return CAQR_ERR_CUDA;
+        const size_t wb = caqr_workspace_bytes(mc, n, dtype, opts);
+        if (S == 1) return factor_impl<T>(mc, n, A + r0, lda, R, ldr, wsb + off, wb, opts, s, dtype);
+        rc = factor_impl<T>(mc, n, A + r0, lda, Rs + (int64_t)c * n, ld, wsb + off, wb, opts, s, dtype);
+    }
+    if (rc) return rc;
+    return combine_impl<T>(S, n, Rs, ld, R, ldr, wsb + cw_off, caqr_combine_workspace_bytes(S, n, dtype), s,
+                           dtype);
+}
+
 extern "C" {
 
 size_t caqr_workspace_bytes(int64_t m, int64_t n, int dtype, const caqr_opts* opts) {
@@ -1390,6 +1500,36 @@ int caqr_set_identity_f32(int64_t m, int64_t n, float* Q, int64_t ldq, caqr_stre
 }
 int caqr_set_identity_f64(int64_t m, int64_t n, double* Q, int64_t ldq, caqr_stream_t stream) {
     return set_identity_impl<double>(m, n, Q, ldq, (cudaStream_t)stream);
+}
+
+size_t caqr_factor_host_workspace_bytes(int64_t m, int64_t n, int chunks, int dtype, const caqr_opts* opts) {
+    int64_t r0, mc;
+    size_t off;
+    return host_layout(m, n, chunks, dtype, opts, 0, &r0, &mc, &off);
+}
+int caqr_factor_host_layout(int64_t m, int64_t n, int chunks, int dtype, const caqr_opts* opts, int c,
+                            int64_t* out3) {
+    if (!out3) return -7;
+    if (c < 0 || c > chunks + 1) return -6;
+    int64_t r0 = 0, mc = 0;
+    size_t off = 0;
+    if (host_layout(m, n, chunks, dtype, opts, c, &r0, &mc, &off) == 0) return -3;
+    out3[0] = r0;
+    out3[1] = mc;
+    out3[2] = (int64_t)off;
+    return 0;
+}
+int caqr_factor_host_f32(int64_t m, int64_t n, int chunks, const float* A_host, int64_t lda_host, float* A,
+                         int64_t lda, float* R, int64_t ldr, void* ws, size_t ws_bytes, const caqr_opts* opts,
+                         caqr_stream_t stream) {
+    return factor_host_impl<float>(m, n, chunks, A_host, lda_host, A, lda, R, ldr, ws, ws_bytes, opts, stream,
+                                   CAQR_F32);
+}
+int caqr_factor_host_f64(int64_t m, int64_t n, int chunks, const double* A_host, int64_t lda_host, double* A,
+                         int64_t lda, double* R, int64_t ldr, void* ws, size_t ws_bytes, const caqr_opts* opts,
+                         caqr_stream_t stream) {
+    return factor_host_impl<double>(m, n, chunks, A_host, lda_host, A, lda, R, ldr, ws, ws_bytes, opts, stream,
+                                    CAQR_F64);
 }
 
 }  // extern "C"

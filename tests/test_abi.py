@@ -142,3 +142,39 @@ def test_info_codes_application_layer_without_gpu(L):
     # caqr_set_identity_f32(m, n, Q, ldq, stream)
     i = L.caqr_set_identity_f32
     assert i(4, 5, one, 4, null) == -2 and i(4, 2, one, 3, null) == -4 and i(4, 2, null, 4, null) == -3
+
+
+def test_factor_host_layout(L):
+    """caqr_factor_host_*: chunk rows m*c/S, 256-B aligned chunk workspaces,
+    then the R stack and the combine workspace (include/caqr.h)."""
+    a256 = lambda x: -(-x // 256) * 256
+    m, n, S = 1_000_003, 192, 8
+    off = 0
+    for c in range(S):
+        r0, mc, o = caqr.caqr_factor_host_layout(m, n, S, c)
+        assert (r0, mc, o) == (m * c // S, m * (c + 1) // S - m * c // S, off)
+        off += a256(caqr.caqr_workspace_bytes(mc, n))
+    assert caqr.caqr_factor_host_layout(m, n, S, S) == (0, S * n, off)
+    off += a256(S * n * n * 4)
+    assert caqr.caqr_factor_host_layout(m, n, S, S + 1) == (0, 0, off)
+    total = off + a256(caqr.caqr_combine_workspace_bytes(S, n))
+    assert caqr.caqr_factor_host_workspace_bytes(m, n, S) == total
+    # S = 1: one chunk = the whole matrix
+    assert caqr.caqr_factor_host_layout(5000, 16, 1, 0) == (0, 5000, 0)
+    # illegal: m/S < n, n > 256 with S > 1, S out of range, bad dtype
+    assert caqr.caqr_factor_host_workspace_bytes(100, 64, 4) == 0
+    assert caqr.caqr_factor_host_workspace_bytes(100_000, 300, 2) == 0
+    assert caqr.caqr_factor_host_workspace_bytes(100_000, 30, 0) == 0
+    assert caqr.caqr_factor_host_workspace_bytes(100_000, 30, 1025) == 0
+    assert caqr.caqr_factor_host_workspace_bytes(100_000, 30, 2, 7) == 0
+    with pytest.raises(caqr.CaqrError):
+        caqr.caqr_factor_host_layout(m, n, S, S + 2)
+    # info codes that need no device: bad m, n, chunks, lda_host, lda, ldr
+    fn = L.caqr_factor_host_f32
+    assert fn(-1, 4, 2, None, 10, None, 10, None, 4, None, 0, None, None) == -1
+    assert fn(10, 11, 2, None, 10, None, 10, None, 11, None, 0, None, None) == -2
+    assert fn(100, 64, 4, None, 100, None, 100, None, 64, None, 0, None, None) == -3
+    assert fn(100, 4, 2, None, 99, None, 100, None, 4, None, 0, None, None) == -5
+    assert fn(100, 4, 2, None, 100, None, 99, None, 4, None, 0, None, None) == -7
+    assert fn(100, 4, 2, None, 100, None, 100, None, 3, None, 0, None, None) == -9
+    assert fn(0, 0, 1, None, 1, None, 1, None, 1, None, 0, None, None) == 0

@@ -567,3 +567,55 @@ def test_sharded_form_q_emulated(caqr, m, n, P, dtype):
     if rows == m:
         Ro = oracle.normalize_signs(oracle.qr(A64, want_q=False, acc=bd["acc"]))
         assert np.linalg.norm(oracle.normalize_signs(R) - Ro) / np.linalg.norm(Ro) <= bd["r"]
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64], ids=["f32", "f64"])
+@pytest.mark.parametrize("m,n,S", [(5000, 16, 1), (20011, 64, 4), (30000, 192, 7), (4099, 33, 3)])
+def test_factor_host_matches_oracle(caqr, m, n, S, dtype):
+    """caqr_factor_host: chunked H2D + per-chunk TSQR + combine (the distributed
+    TSQR tree of P:L181-188 over row blocks of one GPU).  R against the oracle;
+    Q^T A = [R; 0] through the chunk layout (apply_qt per chunk, then the
+    combine's Q^T on the chunks' top n rows)."""
+    A = workloads.gaussian(m, n, seed=m + n + S, dtype=dtype)
+    tdt = torch.float32 if dtype == np.float32 else torch.float64
+    Ah = torch.empty((n, m), dtype=tdt, pin_memory=True).t()
+    Ah.copy_(torch.from_numpy(A))
+    Ad, R, ws = caqr.caqr_factor_host(Ah, S)
+    torch.cuda.synchronize()
+    R = R.cpu().numpy().astype(np.float64)
+    bd = BOUNDS[dtype]
+    assert np.all(np.tril(R, -1) == 0)
+    Ro = oracle.normalize_signs(oracle.qr(A.astype(np.float64), want_q=False, acc=bd["acc"]))
+    assert np.linalg.norm(oracle.normalize_signs(R) - Ro) / np.linalg.norm(Ro) <= bd["r"]
+    code = caqr.CAQR_F32 if dtype == np.float32 else caqr.CAQR_F64
+    C = to_dev(caqr, A)
+    tops = []
+    for c in range(S):
+        r0, mc, off = caqr.caqr_factor_host_layout(m, n, S, c, code)
+        assert mc >= n and r0 == (m * c) // S
+        wb = caqr.caqr_workspace_bytes(mc, n, code)
+        caqr.caqr_apply_qt(Ad[r0:r0 + mc], ws[off:off + wb], C[r0:r0 + mc], n=n)
+        tops.append(C[r0:r0 + n].clone())
+    if S > 1:
+        _, rows, rs_off = caqr.caqr_factor_host_layout(m, n, S, S, code)
+        _, _, cw_off = caqr.caqr_factor_host_layout(m, n, S, S + 1, code)
+        esz = 4 if dtype == np.float32 else 8
+        Rs = ws[rs_off:rs_off + rows * n * esz].view(tdt).view(n, rows).t()
+        st = caqr.colmajor(torch.cat(tops, 0))
+        caqr.caqr_combine_apply(Rs, S, ws[cw_off:], st, trans=True)
+        top = st.cpu().numpy().astype(np.float64)
+    else:
+        top = C.cpu().numpy().astype(np.float64)
+    tol = 50 * bd["res"] * np.abs(R).max()
+    np.testing.assert_allclose(top[:n], R, atol=tol)
+    assert np.abs(top[n:]).max() <= tol
+    # the host factorization's R equals the single-shot device factorization's R up to rounding
+    R1, _, _, _ = gpu_qr(caqr, A, want_q=False)
+    assert np.linalg.norm(oracle.normalize_signs(R1) - oracle.normalize_signs(R)) / np.linalg.norm(R1) <= bd["r"]
+
+
+def test_factor_host_errors(caqr):
+    with pytest.raises(caqr.CaqrError):
+        caqr.caqr_factor_host(torch.zeros(64, 100).t(), 4)  # 100 x 64 in 4 chunks: m/S < n
+    with pytest.raises(ValueError):
+        caqr.caqr_factor_host(torch.zeros(100, 4, device="cuda").t().contiguous().t(), 2)
