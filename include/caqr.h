@@ -24,11 +24,13 @@
  * Conventions for every entry point:
  *   - Matrices are column-major with a leading dimension ("originally
  *     stored in column major order").  ALL matrix and workspace pointers are
- *     DEVICE pointers (cudaMalloc'd or torch CUDA storage) on the current device.
+ *     DEVICE pointers (cudaMalloc'd or torch CUDA storage) on the current device,
+ *     except A_host of caqr_factor_host_* (host memory, by name).
  *   - Calls only enqueue work on `stream` (0 = legacy default stream); they never
  *     synchronise the device, never allocate device memory, and are safe to
  *     capture into a CUDA graph.  They are reentrant; the only process state is
- *     a lazily-filled per-device attribute cache.
+ *     a lazily-filled per-device attribute cache and the lazily-created side
+ *     stream (CAQR early start) and copy stream (caqr_factor_host_*) per device.
  *   - Return value: LAPACK "info".  0 = success; -i = argument i is illegal (the
  *     call does nothing); CAQR_ERR_CUDA (1) = a CUDA launch failed (see
  *     caqr_last_cuda_error); CAQR_ERR_NCCL (2) = an NCCL call failed.
@@ -183,7 +185,9 @@ int caqr_combine_apply_f64(int P, int64_t n, const double *Rstack, int64_t ld, c
  * of the combine workspace}: with them, caqr_apply_qt_* per chunk followed by
  * caqr_combine_apply_* on the chunks' top n rows applies Q^T (as for the
  * row-sharded multi-GPU factorization).  The caller keeps A_host unchanged
- * until the stream reaches the end of the call.  Layout query: 0, or -3 (bad
+ * until the stream reaches the end of the call.  Calls from several host
+ * threads are serialised while they issue (shared copy stream and events).
+ * Layout query: 0, or -3 (bad
  * m, n, chunks, dtype, opts), -6 (c out of range), -7 (out3 NULL).
  * caqr_factor_host_workspace_bytes returns 0 on illegal arguments. */
 size_t caqr_factor_host_workspace_bytes(int64_t m, int64_t n, int chunks, int dtype, const caqr_opts *opts);

@@ -1139,6 +1139,11 @@ static int factor_host_impl(int64_t m, int64_t n, int S, const T* Ah, int64_t ld
     cudaStream_t cs;
     cudaEvent_t* ev;
     if (!copy_stream(&cs, &ev)) return CAQR_ERR_CUDA;
+    // The copy stream and its events are shared per process: calls from
+    // several host threads issue one at a time (each wait binds to its own
+    // call's event records).
+    static std::mutex issue_mu;
+    std::lock_guard<std::mutex> issue_lock(issue_mu);
     // The copies may overwrite A only after the work already queued on s.
     if (cudaEventRecord(ev[S], s) != cudaSuccess || cudaStreamWaitEvent(cs, ev[S], 0) != cudaSuccess)
         return CAQR_ERR_CUDA;
