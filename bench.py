@@ -382,6 +382,35 @@ def main():
                "serial": {"value": flops / (serial_ms * 1e-3) / 1e9, "ms_per_step": serial_ms,
                           "api": "whole pinned H2D, then caqr_factor, + D2H(R)"}}
         del hws
+    elif not args.no_e2e:
+        # N > 1: each rank's pinned host shard -> H2D, the distributed factor
+        # (local TSQR + NCCL all-gather of the R's + combine), D2H of R; the
+        # per-step time is the max over ranks.
+        Ah = torch.empty((n, m), dtype=tdt, pin_memory=True).t()
+        Ah.copy_(A0)
+        Rh = torch.empty((n, n), dtype=tdt, pin_memory=True)
+        torch.cuda.synchronize()
+        ee = []
+        for i in range(max(3, min(args.steps, 10)) + 2):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            flush.zero_()
+            dist.barrier()
+            torch.cuda.synchronize()
+            a.record(stream)
+            A.copy_(Ah, non_blocking=True)
+            step()
+            Rh.copy_(R, non_blocking=True)
+            b.record(stream)
+            torch.cuda.synchronize()
+            if i >= 2:
+                ee.append(a.elapsed_time(b))
+        t = torch.tensor([sum(ee) / len(ee)], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_ms = float(t.item())
+        e2e = {"value": flops / (e2e_ms * 1e-3) / 1e9, "unit": UNIT, "ms_per_step": e2e_ms,
+               "h2d_bytes_per_step": m_total * n * esz, "d2h_bytes_per_step": world * n * n * esz,
+               "api": "per rank: pinned H2D of the row shard + caqr_dist_factor (local TSQR, NCCL all-gather "
+                      "of the R's, combine) + D2H(R); max over ranks"}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
