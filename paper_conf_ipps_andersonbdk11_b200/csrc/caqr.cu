@@ -1099,21 +1099,32 @@ static size_t host_layout(int64_t m, int64_t n, int S, int dtype, const caqr_opt
 }
 
 // One copy stream and a pool of events per device for the H2D pipeline.
-static bool copy_stream(cudaStream_t* cs, cudaEvent_t** evs) {
+// (plus a second compute stream: consecutive chunks' TSQRs alternate between
+// the caller's stream and it, so one chunk's latency-bound tree tail overlaps
+// the next chunk's leaves).
+static bool copy_stream(cudaStream_t* cs, cudaStream_t* s2, cudaEvent_t** evs) {
     static std::mutex mu;
-    static cudaStream_t streams[64] = {};
-    static cudaEvent_t pool[64][1025] = {};
+    static cudaStream_t streams[64][2] = {};
+    static cudaEvent_t pool[64][1027] = {};
     int dev = 0;
     if (cudaGetDevice(&dev) != cudaSuccess || dev >= 64) return false;
     std::lock_guard<std::mutex> lk(mu);
-    if (!streams[dev]) {
-        if (cudaStreamCreateWithFlags(&streams[dev], cudaStreamNonBlocking) != cudaSuccess) return false;
-        for (int i = 0; i < 1025; ++i)
+    if (!streams[dev][0]) {
+        if (cudaStreamCreateWithFlags(&streams[dev][0], cudaStreamNonBlocking) != cudaSuccess ||
+            cudaStreamCreateWithFlags(&streams[dev][1], cudaStreamNonBlocking) != cudaSuccess)
+            return false;
+        for (int i = 0; i < 1027; ++i)
             if (cudaEventCreateWithFlags(&pool[dev][i], cudaEventDisableTiming) != cudaSuccess) return false;
     }
-    *cs = streams[dev];
+    *cs = streams[dev][0];
+    *s2 = streams[dev][1];
     *evs = pool[dev];
     return true;
+}
+
+static inline bool host_dual_policy() {
+    const char* e = getenv("CAQR_HOST_DUAL");
+    return !(e && e[0] == '0');
 }
 
 template <typename T>
@@ -1136,16 +1147,18 @@ static int factor_host_impl(int64_t m, int64_t n, int S, const T* Ah, int64_t ld
     if (!R) return -8;
     if (!ws) return -10;
     if (ws_bytes < need) return -11;
-    cudaStream_t cs;
+    cudaStream_t cs, s2;
     cudaEvent_t* ev;
-    if (!copy_stream(&cs, &ev)) return CAQR_ERR_CUDA;
+    if (!copy_stream(&cs, &s2, &ev)) return CAQR_ERR_CUDA;
     // The copy stream and its events are shared per process: calls from
     // several host threads issue one at a time (each wait binds to its own
     // call's event records).
     static std::mutex issue_mu;
     std::lock_guard<std::mutex> issue_lock(issue_mu);
     // The copies may overwrite A only after the work already queued on s.
-    if (cudaEventRecord(ev[S], s) != cudaSuccess || cudaStreamWaitEvent(cs, ev[S], 0) != cudaSuccess)
+    const bool dual = S > 1 && host_dual_policy();
+    if (cudaEventRecord(ev[S], s) != cudaSuccess || cudaStreamWaitEvent(cs, ev[S], 0) != cudaSuccess ||
+        (dual && cudaStreamWaitEvent(s2, ev[S], 0) != cudaSuccess))
         return CAQR_ERR_CUDA;
     char* wsb = static_cast<char*>(ws);
     for (int c = 0; c < S; ++c) {
@@ -1166,12 +1179,15 @@ static int factor_host_impl(int64_t m, int64_t n, int S, const T* Ah, int64_t ld
     int rc = 0;
     for (int c = 0; c < S && !rc; ++c) {
         host_layout(m, n, S, dtype, opts, c, &r0, &mc, &off);
-        if (cudaStreamWaitEvent(s, ev[c], 0) != cudaSuccess) return CAQR_ERR_CUDA;
+        cudaStream_t sc = dual && (c & 1) ? s2 : s;
+        if (cudaStreamWaitEvent(sc, ev[c], 0) != cudaSuccess) return CAQR_ERR_CUDA;
         const size_t wb = caqr_workspace_bytes(mc, n, dtype, opts);
         if (S == 1) return factor_impl<T>(mc, n, A + r0, lda, R, ldr, wsb + off, wb, opts, s, dtype);
-        rc = factor_impl<T>(mc, n, A + r0, lda, Rs + (int64_t)c * n, ld, wsb + off, wb, opts, s, dtype);
+        rc = factor_impl<T>(mc, n, A + r0, lda, Rs + (int64_t)c * n, ld, wsb + off, wb, opts, sc, dtype);
     }
     if (rc) return rc;
+    if (dual && (cudaEventRecord(ev[S + 1], s2) != cudaSuccess || cudaStreamWaitEvent(s, ev[S + 1], 0) != cudaSuccess))
+        return CAQR_ERR_CUDA;
     return combine_impl<T>(S, n, Rs, ld, R, ldr, wsb + cw_off, caqr_combine_workspace_bytes(S, n, dtype), s,
                            dtype);
 }

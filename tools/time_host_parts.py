@@ -24,7 +24,7 @@ Ah = torch.empty((n, m), pin_memory=True).t()
 Ah.copy_(torch.randn(m, n))
 A = caqr.colmajor_empty(m, n)
 print(f"H2D whole {ev_time(lambda: A.copy_(Ah, non_blocking=True)):.3f} ms")
-for S in (8, 12, 16, 24, 32):
+for S in (8, 12, 16, 24, 32, 48):
     mc = m // S
     Ac = caqr.colmajor_empty(mc, n)
     Ac.copy_(Ah[:mc])
