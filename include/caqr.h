@@ -30,7 +30,8 @@
  *     synchronise the device, never allocate device memory, and are safe to
  *     capture into a CUDA graph.  They are reentrant; the only process state is
  *     a lazily-filled per-device attribute cache and the lazily-created side
- *     stream (CAQR early start) and copy stream (caqr_factor_host_*) per device.
+ *     stream (CAQR early start) and copy + second compute stream
+ *     (caqr_factor_host_*) per device.
  *   - Return value: LAPACK "info".  0 = success; -i = argument i is illegal (the
  *     call does nothing); CAQR_ERR_CUDA (1) = a CUDA launch failed (see
  *     caqr_last_cuda_error); CAQR_ERR_NCCL (2) = an NCCL call failed.
@@ -162,7 +163,9 @@ int caqr_combine_apply_f64(int P, int64_t n, const double *Rstack, int64_t ld, c
  * A = QR of a matrix that lives in HOST memory (pinned for overlap).  The rows
  * are split into `chunks` row blocks, chunk c = rows [m*c/chunks,
  * m*(c+1)/chunks); each block's H2D copy runs on a copy engine (a library copy
- * stream) while the previous blocks are factored on `stream` by caqr_factor_*;
+ * stream) while the previous blocks are factored by caqr_factor_* (odd chunks
+ * on a second library stream joined back into `stream`, CAQR_HOST_DUAL=0: all
+ * on `stream`);
  * the chunks' R factors are then reduced by caqr_combine_* — the extra tree
  * level of the distributed TSQR the paper cites, here with row
  * blocks of one GPU as its leaves.  Not in the paper (its runtimes exclude the
