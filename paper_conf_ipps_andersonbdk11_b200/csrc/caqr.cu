@@ -14,6 +14,7 @@
 
 #include "../../include/caqr.h"
 #include "tsqr_fused.cuh"
+#include "tsqr_chain.cuh"
 #include "tsqr_kernels.cuh"
 #include "tsqr_skinny.cuh"
 #include "rpca.cuh"
@@ -29,11 +30,12 @@ static thread_local int g_last_cuda_error = 0;
 enum KernelId { K_PANEL_FACTOR = 0, K_PANEL_UPDATE = 1, K_EXTRACT_R = 2, K_SET_IDENTITY = 3,
                 K_TSQR_FUSED = 4, K_TSQR_SKINNY = 5, K_SVD_SMALL = 6, K_SVT_CORE = 7, K_EMBED_TOP = 8,
                 K_RPCA_UPDATE = 9, K_RPCA_INIT = 10, K_ABSMAX = 11, K_CHAIN_UPDATE = 12, K_STREAM_APPLY = 13,
-                K_TRSM = 14, K_NUM = 15 };
+                K_TRSM = 14, K_TSQR_CHAIN = 15, K_NUM = 16 };
 static const char* const kKernelNames[K_NUM] = {"panel_factor", "panel_update", "extract_r", "set_identity",
                                                 "tsqr_fused",   "tsqr_skinny",  "svd_small", "svt_core",
                                                 "embed_top",    "rpca_update",  "rpca_init", "absmax",
-                                                "node_update",  "stream_apply", "trsm_upper"};
+                                                "node_update",  "stream_apply", "trsm_upper",
+                                                "tsqr_chain"};
 struct Trace {
     std::mutex mu;
     bool on = false;
@@ -82,9 +84,20 @@ struct Plan {
     int64_t ngroups = 0;
     int64_t chain_target = 296;  // chains per group (tree leaves)
     bool skinny = false;         // warp-per-task skinny kernel (fp32, n <= 16)
+    bool chain = false;          // chain kernel + merge-only fused tree (fp32, 16 < n <= 256)
 };
 
 static inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+// Chain kernel policy (CAQR_CHAIN=1: the chain kernel does the chains, the
+// fused kernel the tree; default: the fused kernel does both) and its tile height: 128 / 192 / 256 rows (>= n: the chain R lives in
+// the first tile's top n rows).  Read per call so tests can compare paths.
+static inline bool chain_policy() {
+    const char* e = getenv("CAQR_CHAIN");
+    return e && e[0] == '1';
+}
+static inline int64_t chain_tile_rows(int64_t n) { return n <= 128 ? 128 : (n <= 192 ? 192 : 256); }
+constexpr int64_t kChainTarget2 = 444;  // chains: 3 per B200 SM (device-independent constant)
 static inline int64_t round_up(int64_t a, int64_t b) { return ceil_div(a, b) * b; }
 
 // Returns 0, or the info code of the offending argument position `opt_pos`.
@@ -110,7 +123,13 @@ static int make_plan(int64_t m, int64_t n, int dtype, const caqr_opts* o, int op
     pl->chain_target = pl->skinny ? (s16 ? 2 * kStreamChains : kStreamChains) : kChainTarget;
     if (const char* e = getenv("CAQR_CHAIN_TARGET"))  // diagnostics: chains per group (tile sweep)
         pl->chain_target = std::max<int64_t>(1, atoll(e));
+    // fp32 whole-width groups (16 < n <= 256): the chain kernel (tsqr_chain.cuh),
+    // tiles of 128 / 192 / 256 rows (>= n), ~3 chains per SM
+    pl->chain = dtype == CAQR_F32 && !pl->skinny && nb == n && n > 16 && n <= 256 && chain_policy() &&
+                !(o && o->leaf_rows > 0 && o->leaf_rows != chain_tile_rows(n));
+    if (pl->chain && !getenv("CAQR_CHAIN_TARGET")) pl->chain_target = kChainTarget2;
     int64_t b = (o && o->leaf_rows > 0) ? o->leaf_rows
+                                        : pl->chain ? chain_tile_rows(n)
                                         : (pl->skinny ? (n <= 8 && !s16 ? 256 : 128)
                                                       : (nb <= kFusedLeaf ? kFusedLeaf : kMaxLeaf));
     if (b % 32 != 0 || b > kMaxLeaf) return -opt_pos;
@@ -678,8 +697,59 @@ static int launch_stream(const Geom& G, T* A, T* Tws, int* sync, cudaStream_t s,
     return 0;
 }
 
+// Chain phase of a whole-width fp32 group (tsqr_chain.cuh): one persistent
+// launch over the P chains; the tree over their slots follows (merge-only
+// fused kernel).
+template <int NQ, int SEG, int MINB>
+static cudaError_t launch_chain_cfg(const Geom& G, float* A, float* Tws, int* sync, cudaStream_t s) {
+    const size_t smem = chain_smem_bytes<NQ, SEG>();
+    cudaError_t e = allow_smem(tsqr_chain_kernel<NQ, SEG, MINB>, smem);
+    int occ = 1;
+    if (e == cudaSuccess)
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, tsqr_chain_kernel<NQ, SEG, MINB>, 32 * NQ, smem);
+    if (e != cudaSuccess) return e;
+    const int64_t grid = std::min<int64_t>(G.P, (int64_t)std::max(occ, 1) * num_sms());
+    unsigned long long* prof = prof_buffer();
+    tsqr_chain_kernel<NQ, SEG, MINB><<<(unsigned)grid, 32 * NQ, smem, s>>>(G, A, Tws, sync, prof);
+    return cudaGetLastError();
+}
+
 template <typename T>
-static int factor_group(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, cudaStream_t s) {
+static int launch_chain(const Geom& G, T* A, T* Tws, int* sync, cudaStream_t s, bool* done) {
+    *done = false;
+    if constexpr (sizeof(T) == 4) {
+        if (G.ncols <= 16 || G.ncols > G.b || !(G.b == 128 || G.b == 192 || G.b == 256)) return 0;
+        cudaError_t e = cudaMemsetAsync(sync, 0, group_sync_bytes(G), s);
+        if (e == cudaSuccess) {
+            double fl = 0, by = 0;
+            if (g_trace.on) {
+                const double mr = (double)G.mrows, nc = (double)G.ncols;
+                fl = 2.0 * mr * nc * nc - 2.0 / 3.0 * nc * nc * nc;
+                by = 2.0 * mr * nc * sizeof(T);
+            }
+            TraceScope ts(K_TSQR_CHAIN, fl, by, s);
+            e = G.b == 128   ? launch_chain_cfg<4, 32, 3>(G, A, Tws, sync, s)
+                : G.b == 192 ? launch_chain_cfg<4, 48, 3>(G, A, Tws, sync, s)
+                             : launch_chain_cfg<4, 64, 2>(G, A, Tws, sync, s);
+        }
+        if (e != cudaSuccess) {
+            g_last_cuda_error = (int)e;
+            return CAQR_ERR_CUDA;
+        }
+        *done = true;
+    }
+    return 0;
+}
+
+template <typename T>
+static int factor_group(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, cudaStream_t s,
+                        bool chain = false) {
+    if (chain && do_leaves && fused_ok(G)) {
+        bool done = false;
+        int rc = launch_chain<T>(G, A, Tws, sync, s, &done);
+        if (rc) return rc;
+        if (done) return launch_fused<T>(G, A, Tws, sync, false, s);  // tree over the chain slots
+    }
     if (fused_policy() && do_leaves && G.npan == 1 && G.ncols <= 16 && skinny_policy() == 1) {
         bool done = false;
         const int rc = launch_stream<T>(G, A, Tws, sync, s, &done);
@@ -818,7 +888,7 @@ static int factor_impl(int64_t m, int64_t n, T* A, int64_t lda, T* R, int64_t ld
         int* sync;
         group_ptrs(g, &Tws, &sync);
         if (!overlap || g == 0) {
-            rc = factor_group<T>(G, A, Tws, sync, true, s);
+            rc = factor_group<T>(G, A, Tws, sync, true, s, pl.chain);
         } else if (cudaStreamWaitEvent(s, ev_done, 0) != cudaSuccess) {  // TSQR_g ran on s2
             rc = CAQR_ERR_CUDA;
         }
