@@ -1,3 +1,4 @@
+#include <cstdio>
 // caqr.cu -- host planner + C ABI of libcaqr.so (declared in include/caqr.h).
 //
 // The host side is the paper's "CPU coordinates the GPU's actions and updates
@@ -700,18 +701,52 @@ static int launch_stream(const Geom& G, T* A, T* Tws, int* sync, cudaStream_t s,
 // Chain phase of a whole-width fp32 group (tsqr_chain.cuh): one persistent
 // launch over the P chains; the tree over their slots follows (merge-only
 // fused kernel).
+static inline bool chain_tc_policy() {  // CAQR_CHAIN_TC=0: mma.sync trailing update in the chain kernel
+    const char* e = getenv("CAQR_CHAIN_TC");
+    return !(e && e[0] == '0');
+}
+template <int NQ, int SEG, int MINB, bool TC>
+static cudaError_t launch_chain_cfg(const Geom& G, float* A, float* Tws, int* sync, cudaStream_t s) {
+    const size_t smem = TC ? ChainCfgTC<NQ, SEG>::BYTES : ChainCfg<NQ, SEG>::BYTES;
+    auto kern = tsqr_chain_kernel<NQ, SEG, MINB, TC>;
+    cudaError_t e = allow_smem(kern, smem);
+    int occ = 1;
+    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, 32 * NQ, smem);
+    if (e != cudaSuccess) return e;
+    if (TC) {
+        // The occupancy API counts a tcgen05 kernel as one CTA per SM; the
+        // CTAs co-reside as long as their TMEM allocations (128 columns each)
+        // and registers / shared memory fit.
+        cudaFuncAttributes fa;
+        if (cudaFuncGetAttributes(&fa, kern) == cudaSuccess) {
+            const int by_smem = (int)((228 * 1024) / (smem + fa.sharedSizeBytes + 1024));
+            const int by_regs = 65536 / (((fa.numRegs * 32 + 255) / 256) * 256 * NQ);
+            occ = std::max(1, std::min(4, std::min(by_smem, by_regs)));
+        }
+    }
+    if (const char* e = getenv("CAQR_CHAIN_OCC")) occ = atoi(e);  // diagnostics
+    const int64_t grid = std::min<int64_t>(G.P, (int64_t)std::max(occ, 1) * num_sms());
+    if (getenv("CAQR_CHAIN_DBG")) {
+        cudaFuncAttributes fa;
+        cudaFuncGetAttributes(&fa, kern);
+        int o2 = 0, o3 = 0, o4 = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o2, kern, 32 * NQ, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o3, kern, 32 * NQ, 40000);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o4, kern, 32 * NQ, 60000);
+        fprintf(stderr,
+                "chain kernel TC=%d NQ=%d SEG=%d smem=%zu occ=%d grid=%lld P=%lld K=%lld regs=%d static=%zu "
+                "maxdyn=%d occ(0)=%d occ(40k)=%d occ(60k)=%d\n",
+                (int)TC, NQ, SEG, smem, occ, (long long)grid, (long long)G.P, (long long)G.K, fa.numRegs,
+                fa.sharedSizeBytes, fa.maxDynamicSharedSizeBytes, o2, o3, o4);
+    }
+    unsigned long long* prof = prof_buffer();
+    kern<<<(unsigned)grid, 32 * NQ, smem, s>>>(G, A, Tws, sync, prof);
+    return cudaGetLastError();
+}
 template <int NQ, int SEG, int MINB>
 static cudaError_t launch_chain_cfg(const Geom& G, float* A, float* Tws, int* sync, cudaStream_t s) {
-    const size_t smem = chain_smem_bytes<NQ, SEG>();
-    cudaError_t e = allow_smem(tsqr_chain_kernel<NQ, SEG, MINB>, smem);
-    int occ = 1;
-    if (e == cudaSuccess)
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, tsqr_chain_kernel<NQ, SEG, MINB>, 32 * NQ, smem);
-    if (e != cudaSuccess) return e;
-    const int64_t grid = std::min<int64_t>(G.P, (int64_t)std::max(occ, 1) * num_sms());
-    unsigned long long* prof = prof_buffer();
-    tsqr_chain_kernel<NQ, SEG, MINB><<<(unsigned)grid, 32 * NQ, smem, s>>>(G, A, Tws, sync, prof);
-    return cudaGetLastError();
+    return chain_tc_policy() ? launch_chain_cfg<NQ, SEG, MINB, true>(G, A, Tws, sync, s)
+                             : launch_chain_cfg<NQ, SEG, MINB, false>(G, A, Tws, sync, s);
 }
 
 template <typename T>

@@ -32,7 +32,10 @@
 // ~60 KB shared memory) give 3 chains per SM instead of 2, and the per-column
 // critical path carries no multi-value warp reductions.
 #pragma once
+#include <type_traits>
+#include <cuda_fp16.h>
 #include "tsqr_fused.cuh"
+#include "umma.cuh"
 
 namespace caqr {
 
@@ -201,10 +204,10 @@ __device__ __forceinline__ void chain_build_t(const float* Gs, const float* taus
     for (int j = 0; j < 32; ++j) __stcg(tb + j * 32 + lane, row[j]);  // column-major, coalesced across lanes
 }
 
-// W2(32 x CW) = T^T W (T upper triangular), 3xTF32 mma.sync, one 16 x 8 tile per warp.
-template <class Cfg>
-__device__ __forceinline__ void chain_gemm_tw(const float* Ts, const float* Ws, float* W2s) {
-    constexpr int HS = Cfg::HS, WS = Cfg::WS;
+// W2(32 x 16) = T^T W (T upper triangular), 3xTF32 mma.sync, one 16 x 8 tile per
+// warp (4 warps); strides of T and of W / W2 given.
+template <int HS, int WS>
+__device__ __forceinline__ void chain_gemm_tw_s(const float* Ts, const float* Ws, float* W2s) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int g = lane >> 2, t = lane & 3;
     const int mt = warp & 1, nt = warp >> 1;
@@ -227,6 +230,10 @@ __device__ __forceinline__ void chain_gemm_tw(const float* Ts, const float* Ws, 
     W2s[i0 * WS + c0 + 1] = acc[1];
     W2s[(i0 + 8) * WS + c0] = acc[2];
     W2s[(i0 + 8) * WS + c0 + 1] = acc[3];
+}
+template <class Cfg>
+__device__ __forceinline__ void chain_gemm_tw(const float* Ts, const float* Ws, float* W2s) {
+    chain_gemm_tw_s<Cfg::HS, Cfg::WS>(Ts, Ws, W2s);
 }
 
 // Cs(B x CW) -= V(B x 32) W2(32 x CW) (3xTF32 mma.sync); warp w owns row
@@ -363,33 +370,103 @@ __device__ __forceinline__ void chain_store(const float* Cs, const float* Csl, f
 }
 
 // ---------------------------------------------------------------------------
+// tcgen05 (5th-generation tensor core) trailing update, fp16x2 operands.
+//
+// The three contractions of a node's blocked update -- G = V^T V (for T),
+// W = V^T C and dC = V W2 -- run as tcgen05.mma kind::f16 with fp32 accumulators
+// in tensor memory.  fp32 operands are split x ~ hi + lo (hi = fp16(x), lo =
+// fp16(x - hi)), each with a power-of-two scale: V by 2^15 (|v| <= 1 for a
+// Householder vector with unit head), every column of C and of W2 by 2^e with
+// max|column| * 2^e in [2^14, 2^15).  The 11-bit fp16 significand equals
+// TF32's, so hi + lo carries 22 bits: |x - hi - lo| <= 2^-22 max|column|, the
+// three products hi*hi + hi*lo + lo*hi (exact in fp32, fp32 accumulation)
+// give a normwise error ~2^-21 -- the 3xTF32 bound -- at the
+// storage size of fp32.  One shared buffer holds V as the K-major operand V^T
+// (G, W) and as the MN-major operand V (dC).
+// ---------------------------------------------------------------------------
+template <int NQ, int SEG>
+struct ChainCfgTC {
+    static constexpr int NT = 32 * NQ;
+    static constexpr int NW = NT / 32;
+    static constexpr int B = NQ * SEG;
+    static constexpr int VP = B + 4;
+    static constexpr int CW = 16;
+    static constexpr int HS = 33;
+    static constexpr int WS2 = 17;                     // stride of the 64-row TMEM dumps
+    // floats
+    static constexpr int OFF_V = 0;                    // fp32 Vs[32][VP] / fp16 V hi|lo (64 x B)
+    static constexpr int OFF_C = OFF_V + 32 * VP;      // fp32 C chunk [2][CW][VP]
+    static constexpr int OFF_H = OFF_C + CW * VP;      // Hh[32][HS], then G dump [64][HS] (C buffer 1)
+    static constexpr int OFF_G = OFF_H;
+    static constexpr int OFF_CH = OFF_C + 2 * CW * VP; // fp16 C hi|lo (CW x B each), then W dump [64][WS2]
+    static constexpr int OFF_CS = OFF_CH + CW * B;     // Csl[2][CW][32]
+    static constexpr int OFF_W2H = OFF_CS + 2 * CW * 32;  // fp16 W2 hi|lo (CW x 32 each)
+    static constexpr int OFF_T = OFF_W2H + CW * 32;    // Ts[32][HS]
+    static constexpr int OFF_TAU = OFF_T + 32 * HS;    // taus[32]
+    static constexpr int OFF_SC = OFF_TAU + 32;        // C column scales [CW], W2 column scales [CW]
+    static constexpr int OFF_MB = OFF_SC + 2 * CW;     // mbarrier (8 bytes)
+    static constexpr int FLOATS = OFF_MB + 4;
+    static constexpr size_t BYTES = sizeof(float) * (size_t)FLOATS;
+    static constexpr uint32_t SBO_V = (B / 8) * 128;   // V: byte(i, r) = (i%8)16 + (r%8)2 + (i/8)SBO_V + (r/8)128
+    static constexpr uint32_t SBO_C = (B / 8) * 128;   // C: byte(n, r) likewise
+    static constexpr uint32_t TM_G = 0, TM_W = 32, TM_D1 = 48, TM_D2 = 64;  // TMEM columns
+    static_assert(NQ == 4 && CW * 8 == NT, "layout");
+    static_assert(B % 64 == 0, "row blocks of 128 (+64)");
+    static_assert(OFF_MB % 2 == 0, "mbarrier alignment");
+    static_assert(64 * HS <= CW * VP && 64 * WS2 <= CW * B, "dump areas");
+};
+
+__device__ __forceinline__ float pow2f(int e) { return __uint_as_float((uint32_t)(min(max(e, -126), 127) + 127) << 23); }
+// Scale exponent for a column whose max |value| is m: m * 2^e in [2^14, 2^15).
+__device__ __forceinline__ int col_exp(float m) {
+    return m > 0.f ? 14 - ((int)((__float_as_uint(m) >> 23) & 0xff) - 127) : 0;
+}
+__device__ __forceinline__ void split_f16(float x, __half& h, __half& l) {
+    h = __float2half_rn(x);
+    l = __float2half_rn(x - __half2float(h));
+}
+// pack 4 halves into 8 bytes
+__device__ __forceinline__ uint2 pack4(__half a, __half b, __half c, __half d) {
+    return make_uint2((uint32_t)__half_as_ushort(a) | ((uint32_t)__half_as_ushort(b) << 16),
+                      (uint32_t)__half_as_ushort(c) | ((uint32_t)__half_as_ushort(d) << 16));
+}
+
+// ---------------------------------------------------------------------------
 // The chain kernel.  Grid: persistent CTAs taking chains from sync[0].
 // ---------------------------------------------------------------------------
-template <int NQ, int SEG, int MINB>
+template <int NQ, int SEG, int MINB, bool TC>
 __global__ void __launch_bounds__(32 * NQ, MINB)
 tsqr_chain_kernel(Geom g, float* __restrict__ A, float* __restrict__ Tws, int* __restrict__ sync,
                   unsigned long long* prof) {
-    using Cfg = ChainCfg<NQ, SEG>;
-    constexpr int VP = Cfg::VP, HS = Cfg::HS, WS = Cfg::WS, CW = Cfg::CW;
-    extern __shared__ __align__(16) unsigned char chain_smem_raw[];
+    using Cfg = typename std::conditional<TC, ChainCfgTC<NQ, SEG>, ChainCfg<NQ, SEG>>::type;
+    constexpr int VP = Cfg::VP, HS = Cfg::HS, CW = Cfg::CW;
+    extern __shared__ __align__(128) unsigned char chain_smem_raw[];
     float* sm = reinterpret_cast<float*>(chain_smem_raw);
     float* Vs = sm + Cfg::OFF_V;
     float* Hh = sm + Cfg::OFF_H;
     float* Ts = sm + Cfg::OFF_T;
     float* Gs = sm + Cfg::OFF_G;
-    float* Ws = sm + Cfg::OFF_W;
-    float* W2s = sm + Cfg::OFF_W2;
     float* taus = sm + Cfg::OFF_TAU;
     __shared__ int s_task;
+    __shared__ uint32_t s_tmem;
+    uint32_t mph = 0;  // mbarrier phase (TC)
+    if constexpr (TC) {
+        if (threadIdx.x < 32) umma::tmem_alloc<128>(&s_tmem);
+        if (threadIdx.x == 0) umma::mbar_init(reinterpret_cast<uint64_t*>(sm + Cfg::OFF_MB), 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        umma::fence_before_sync();
+        __syncthreads();
+        umma::fence_after_sync();
+    }
     // optional phase profile (diagnostics, CAQR_PROFILE=1): thread 0's clock
-    __shared__ unsigned long long pacc[7];  // [6] = last stamp
-    if (threadIdx.x < 7) pacc[threadIdx.x] = threadIdx.x == 6 ? (unsigned long long)clock64() : 0ull;
+    __shared__ unsigned long long pacc[11];  // [10] = last stamp
+    if (threadIdx.x < 11) pacc[threadIdx.x] = threadIdx.x == 10 ? (unsigned long long)clock64() : 0ull;
 #define CHAIN_PROF(k)                                 \
     do {                                              \
         if (prof && threadIdx.x == 0) {               \
             const unsigned long long t1_ = clock64(); \
-            pacc[k] += t1_ - pacc[6];                 \
-            pacc[6] = t1_;                            \
+            pacc[k] += t1_ - pacc[10];                \
+            pacc[10] = t1_;                           \
         }                                             \
     } while (0)
 
@@ -566,9 +643,10 @@ tsqr_chain_kernel(Geom g, float* __restrict__ A, float* __restrict__ Tws, int* _
                 CHAIN_PROF(1);
                 // V columns >= wp are zero; a leaf's head-block rows: 1 on the
                 // diagonal, v below, 0 above
+                if constexpr (!TC)
                 for (int jj = wp + (tid / 32); jj < 32; jj += Cfg::NW)
                     for (int r = lane; r < Cfg::B; r += 32) Vs[(size_t)jj * VP + r] = 0.f;
-                if (leaf) {
+                if (!TC && leaf) {
                     for (int e = tid; e < 32 * 32; e += Cfg::NT) {
                         const int k = e & 31, jj = e >> 5;
                         if (jj < wp && hr0 + k < Cfg::B)
@@ -604,11 +682,6 @@ tsqr_chain_kernel(Geom g, float* __restrict__ A, float* __restrict__ Tws, int* _
                         if (jj < wp && i <= jj) A[(c0 + jj) * lda + slot + hr0 + i] = Hh[i * HS + jj];
                     }
                 }
-                __syncthreads();
-                chain_gemm_gram<Cfg>(Vs, Gs);  // G = V^T V (tile part)
-                __syncthreads();
-                if (tid < 32) chain_build_t(Gs, taus, wp, Ts, Tws + (t * g.npan + p) * (kPW * kPW), HS);
-
                 CHAIN_PROF(2);
                 // ---------------- trailing update --------------------------------
                 const int64_t tfirst = c0 + 32, tend = g.col0 + g.ncols;
@@ -621,42 +694,312 @@ tsqr_chain_kernel(Geom g, float* __restrict__ A, float* __restrict__ Tws, int* _
                     *cb = tfirst + (int64_t)CW * k;
                     return (int)min((int64_t)CW, tend - *cb);
                 };
-                if (nchunk > 0) {
-                    int64_t cb;
-                    const int n0c = chunk_cols(cid(0), &cb);
-                    chain_stage<Cfg>(sm + Cfg::OFF_C, sm + Cfg::OFF_CS, A, lda, cb, n0c, s, h, slotp, wp, leaf, hr0);
-                }
-                for (int ib = 0; ib < nchunk; ++ib) {
-                    int64_t cb0;
-                    const int ncb = chunk_cols(cid(ib), &cb0);
-                    float* Cs = sm + Cfg::OFF_C + (ib & 1) * CW * VP;
-                    float* Csl = sm + Cfg::OFF_CS + (ib & 1) * CW * 32;
-                    if (ib + 1 < nchunk) {  // prefetch the next chunk into the other buffer
-                        int64_t cb1;
-                        const int n1c = chunk_cols(cid(ib + 1), &cb1);
-                        chain_stage<Cfg>(sm + Cfg::OFF_C + ((ib + 1) & 1) * CW * VP,
-                                         sm + Cfg::OFF_CS + ((ib + 1) & 1) * CW * 32, A, lda, cb1, n1c, s, h, slotp, wp,
-                                         leaf, hr0);
-                        asm volatile("cp.async.wait_group 1;" ::: "memory");
-                    } else {
-                        asm volatile("cp.async.wait_group 0;" ::: "memory");
+                if constexpr (TC) {
+                    using umma::smem_u32;
+                    uint64_t* mbar = reinterpret_cast<uint64_t*>(sm + Cfg::OFF_MB);
+                    const uint32_t tmem = s_tmem;
+                    unsigned char* Vh = reinterpret_cast<unsigned char*>(sm + Cfg::OFF_V);   // fp16 V hi | lo
+                    unsigned char* Ch = reinterpret_cast<unsigned char*>(sm + Cfg::OFF_CH);  // fp16 C hi | lo
+                    unsigned char* W2h = reinterpret_cast<unsigned char*>(sm + Cfg::OFF_W2H);
+                    float* cscale = sm + Cfg::OFF_SC;
+                    float* wscale = cscale + CW;
+                    const int warp = tid >> 5;
+                    auto wait_mma = [&]() {
+                        umma::mbar_wait(mbar, mph);
+                        mph ^= 1u;
+                        umma::fence_after_sync();
+                    };
+                    // ---- V -> fp16 hi | lo (scaled by 2^15), K-major V^T layout ----
+                    __syncthreads();  // every consumer is done with the fp32 Vs; Hh complete
+                    {
+#pragma unroll
+                        for (int i = 0; i < SEG; i += 4) {
+                            const int r = q * SEG + i;
+                            float v4[4];
+#pragma unroll
+                            for (int e = 0; e < 4; ++e) {
+                                float v = x[i + e];
+                                if (leaf) {
+                                    const int k = r + e - hr0;  // head-block row
+                                    if (k >= 0 && k < 32) v = k > c ? Hh[k * HS + c] : (k == c ? 1.f : 0.f);
+                                }
+                                v4[e] = c < wp ? v * 32768.f : 0.f;
+                            }
+                            __half h0, l0, h1, l1, h2, l2, h3, l3;
+                            split_f16(v4[0], h0, l0);
+                            split_f16(v4[1], h1, l1);
+                            split_f16(v4[2], h2, l2);
+                            split_f16(v4[3], h3, l3);
+                            const uint32_t off = (c % 8) * 16 + (r % 8) * 2 + (c / 8) * Cfg::SBO_V + (r / 8) * 128;
+                            *reinterpret_cast<uint2*>(Vh + off) = pack4(h0, h1, h2, h3);
+                            *reinterpret_cast<uint2*>(Vh + off + 4 * Cfg::SBO_V) = pack4(l0, l1, l2, l3);
+                        }
+                    }
+                    umma::fence_async_smem();
+                    __syncthreads();
+                    // ---- G = V^T V (M = 64: [hi; lo], N = 32, K = B) ----
+                    if (tid == 0) {
+                        umma::fence_after_sync();
+                        const uint32_t id = umma::idesc_f16(64, 32, false, false);
+                        for (int kk = 0; kk < Cfg::B / 16; ++kk)
+                            for (int hl = 0; hl < 2; ++hl) {
+                                const uint64_t ad = umma::sdesc(smem_u32(Vh) + kk * 256, 128, Cfg::SBO_V);
+                                const uint64_t bd =
+                                    umma::sdesc(smem_u32(Vh) + hl * 4 * Cfg::SBO_V + kk * 256, 128, Cfg::SBO_V);
+                                umma::mma_f16(tmem + Cfg::TM_G, ad, bd, id, kk > 0 || hl > 0);
+                            }
+                        umma::commit(mbar);
+                    }
+                    if (nchunk > 0) {  // first chunk's staging overlaps G (Hh / G dump live in C buffer 1)
+                        int64_t cb;
+                        const int n0c = chunk_cols(cid(0), &cb);
+                        chain_stage<Cfg>(sm + Cfg::OFF_C, sm + Cfg::OFF_CS, A, lda, cb, n0c, s, h, slotp, wp, leaf,
+                                         hr0);
+                    }
+                    wait_mma();
+                    {  // TMEM (M = 64 layout: warp w, lanes < 16 = rows 16w + l) -> G dump [64][HS]
+                        float v[16];
+                        const int row = 16 * warp + lane;
+                        umma::tmem_ld16(tmem + ((uint32_t)(32 * warp) << 16) + Cfg::TM_G, v);
+                        if (lane < 16)
+#pragma unroll
+                            for (int j = 0; j < 16; ++j) Gs[row * HS + j] = v[j];
+                        umma::tmem_ld16(tmem + ((uint32_t)(32 * warp) << 16) + Cfg::TM_G + 16, v);
+                        if (lane < 16)
+#pragma unroll
+                            for (int j = 0; j < 16; ++j) Gs[row * HS + 16 + j] = v[j];
                     }
                     __syncthreads();
-                    CHAIN_PROF(3);
-                    chain_gemm_vtc<Cfg>(Vs, Cs, Csl, !leaf, Ws);
+                    for (int e = tid; e < 32 * 32; e += Cfg::NT) {  // G = (hi rows + lo rows) 2^-30
+                        const int i = e >> 5, j = e & 31;
+                        Gs[i * HS + j] = (Gs[i * HS + j] + Gs[(i + 32) * HS + j]) * 0x1p-30f;
+                    }
                     __syncthreads();
-                    chain_gemm_tw<Cfg>(Ts, Ws, W2s);
-                    __syncthreads();
-                    if (!leaf)  // slot rows: C_slot -= W2 (V's head part is the identity)
-                        for (int e = tid; e < CW * 32; e += Cfg::NT) {
-                            const int cc = e >> 5, i = e & 31;
-                            Csl[cc * 32 + i] -= W2s[i * WS + cc];
+                    if (tid < 32) chain_build_t(Gs, taus, wp, Ts, Tws + (t * g.npan + p) * (kPW * kPW), HS);
+                    CHAIN_PROF(2);
+                    // ---- trailing chunks ----
+                    for (int ib = 0; ib < nchunk; ++ib) {
+                        int64_t cb0;
+                        const int ncb = chunk_cols(cid(ib), &cb0);
+                        float* Cs = sm + Cfg::OFF_C + (ib & 1) * CW * VP;
+                        float* Csl = sm + Cfg::OFF_CS + (ib & 1) * CW * 32;
+                        asm volatile("cp.async.wait_group 0;" ::: "memory");
+                        __syncthreads();  // chunk ib staged; previous chunk's epilogue done; T ready
+                        if (ib + 1 < nchunk) {  // prefetch the next chunk into the other buffer
+                            int64_t cb1;
+                            const int n1c = chunk_cols(cid(ib + 1), &cb1);
+                            chain_stage<Cfg>(sm + Cfg::OFF_C + ((ib + 1) & 1) * CW * VP,
+                                             sm + Cfg::OFF_CS + ((ib + 1) & 1) * CW * 32, A, lda, cb1, n1c, s, h, slotp,
+                                             wp, leaf, hr0);
                         }
-                    chain_gemm_update<Cfg>(Vs, Cs, W2s);
+                        CHAIN_PROF(3);
+                        // C -> fp16 hi | lo with a power-of-two scale per column (K-major B of W = V^T C)
+                        {
+                            const int cc = tid >> 3, u0 = tid & 7;
+                            constexpr int NQ4 = Cfg::B / 4;
+                            float vals[(NQ4 + 7) / 8][4];
+                            float m = 0.f;
+#pragma unroll
+                            for (int k2 = 0; k2 < (NQ4 + 7) / 8; ++k2) {
+                                const int u = u0 + 8 * k2;
+                                float4 f = make_float4(0.f, 0.f, 0.f, 0.f);
+                                if (u < NQ4) f = *reinterpret_cast<const float4*>(Cs + (size_t)cc * VP + 4 * u);
+                                vals[k2][0] = f.x;
+                                vals[k2][1] = f.y;
+                                vals[k2][2] = f.z;
+                                vals[k2][3] = f.w;
+                                m = fmaxf(m, fmaxf(fmaxf(fabsf(f.x), fabsf(f.y)), fmaxf(fabsf(f.z), fabsf(f.w))));
+                            }
+                            m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, 1));
+                            m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, 2));
+                            m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, 4));
+                            const int ex = col_exp(m);
+                            const float sc = pow2f(ex);
+                            if (u0 == 0) cscale[cc] = pow2f(-ex - 15);  // unscale of W: 2^-(15+e)
+#pragma unroll
+                            for (int k2 = 0; k2 < (NQ4 + 7) / 8; ++k2) {
+                                const int u = u0 + 8 * k2;
+                                if (u < NQ4) {
+                                    const int r = 4 * u;
+                                    __half h0, l0, h1, l1, h2, l2, h3, l3;
+                                    split_f16(vals[k2][0] * sc, h0, l0);
+                                    split_f16(vals[k2][1] * sc, h1, l1);
+                                    split_f16(vals[k2][2] * sc, h2, l2);
+                                    split_f16(vals[k2][3] * sc, h3, l3);
+                                    const uint32_t off =
+                                        (cc % 8) * 16 + (r % 8) * 2 + (cc / 8) * Cfg::SBO_C + (r / 8) * 128;
+                                    *reinterpret_cast<uint2*>(Ch + off) = pack4(h0, h1, h2, h3);
+                                    *reinterpret_cast<uint2*>(Ch + CW * Cfg::B * 2 + off) = pack4(l0, l1, l2, l3);
+                                }
+                            }
+                        }
+                        umma::fence_async_smem();
+                        __syncthreads();
+                        // ---- W = V^T C (M = 64 [hi; lo] x N = CW, K = B) ----
+                        if (tid == 0) {
+                            umma::fence_after_sync();
+                            const uint32_t id = umma::idesc_f16(64, CW, false, false);
+                            for (int kk = 0; kk < Cfg::B / 16; ++kk)
+                                for (int hl = 0; hl < 2; ++hl) {
+                                    const uint64_t ad = umma::sdesc(smem_u32(Vh) + kk * 256, 128, Cfg::SBO_V);
+                                    const uint64_t bd = umma::sdesc(smem_u32(Ch) + hl * CW * Cfg::B * 2 + kk * 256,
+                                                                    128, Cfg::SBO_C);
+                                    umma::mma_f16(tmem + Cfg::TM_W, ad, bd, id, kk > 0 || hl > 0);
+                                }
+                            umma::commit(mbar);
+                        }
+                        wait_mma();
+                        CHAIN_PROF(6);
+                        float* Wd = sm + Cfg::OFF_CH;  // W dump [64][WS2] over the (consumed) fp16 C
+                        {
+                            float v[16];
+                            umma::tmem_ld16(tmem + ((uint32_t)(32 * warp) << 16) + Cfg::TM_W, v);
+                            __syncwarp();
+                            if (lane < 16)
+#pragma unroll
+                                for (int j = 0; j < 16; ++j) Wd[(16 * warp + lane) * Cfg::WS2 + j] = v[j];
+                        }
+                        __syncthreads();
+                        // W (rows 0..31) = (hi rows + lo rows) / (2^15 scale) (+ C_slot)
+                        for (int e = tid; e < 32 * CW; e += Cfg::NT) {
+                            const int i = e / CW, n = e % CW;
+                            float w = (Wd[i * Cfg::WS2 + n] + Wd[(i + 32) * Cfg::WS2 + n]) * cscale[n];
+                            if (!leaf) w += Csl[n * 32 + i];
+                            Wd[i * Cfg::WS2 + n] = w;
+                        }
+                        __syncthreads();
+                        chain_gemm_tw_s<Cfg::HS, Cfg::WS2>(Ts, Wd, Wd + 32 * Cfg::WS2);  // W2 (rows 32..63 of the dump)
+                        __syncthreads();
+                        // W2 -> C_slot update; fp16 hi | lo with a per-column scale (K-major B of dC = V W2)
+                        {
+                            const int n = tid >> 3, i0 = 4 * (tid & 7);
+                            float w2[4];
+                            float m = 0.f;
+#pragma unroll
+                            for (int u = 0; u < 4; ++u) {
+                                w2[u] = Wd[(32 + i0 + u) * Cfg::WS2 + n];
+                                m = fmaxf(m, fabsf(w2[u]));
+                                if (!leaf) Csl[n * 32 + i0 + u] -= w2[u];
+                            }
+                            m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, 1));
+                            m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, 2));
+                            m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, 4));
+                            const int ex = col_exp(m);
+                            const float sc = pow2f(ex);
+                            if ((tid & 7) == 0) wscale[n] = pow2f(-ex - 15);  // unscale of dC: 2^-(15+e)
+                            __half h0, l0, h1, l1, h2, l2, h3, l3;
+                            split_f16(w2[0] * sc, h0, l0);
+                            split_f16(w2[1] * sc, h1, l1);
+                            split_f16(w2[2] * sc, h2, l2);
+                            split_f16(w2[3] * sc, h3, l3);
+                            const uint32_t off = (n % 8) * 16 + (i0 % 8) * 2 + (n / 8) * 512 + (i0 / 8) * 128;
+                            *reinterpret_cast<uint2*>(W2h + off) = pack4(h0, h1, h2, h3);
+                            *reinterpret_cast<uint2*>(W2h + CW * 32 * 2 + off) = pack4(l0, l1, l2, l3);
+                        }
+                        umma::fence_async_smem();
+                        __syncthreads();
+                        CHAIN_PROF(7);
+                        // ---- dC = V W2 (A = V MN-major, row blocks of 128 (+ 64); 3 products) ----
+                        if (tid == 0) {
+                            umma::fence_after_sync();
+                            constexpr int NB = (Cfg::B + 127) / 128;
+                            for (int mb = 0; mb < NB; ++mb) {
+                                const int mrows = min(128, Cfg::B - 128 * mb);
+                                const uint32_t id = umma::idesc_f16(mrows, CW, true, false);
+                                const uint32_t dcol = mb == 0 ? Cfg::TM_D1 : Cfg::TM_D2;
+                                bool acc = false;
+#pragma unroll
+                                for (int pr = 0; pr < 3; ++pr) {
+                                    const int ah = pr == 2 ? 1 : 0, bh = pr == 1 ? 1 : 0;  // (hi,hi) (hi,lo) (lo,hi)
+                                    for (int kk = 0; kk < 2; ++kk) {
+                                        const uint64_t ad = umma::sdesc(smem_u32(Vh) + mb * 16 * 128 + ah * 4 * Cfg::SBO_V +
+                                                                            kk * 2 * Cfg::SBO_V,
+                                                                        Cfg::SBO_V, 128);
+                                        const uint64_t bd =
+                                            umma::sdesc(smem_u32(W2h) + bh * CW * 32 * 2 + kk * 256, 128, 512);
+                                        umma::mma_f16(tmem + dcol, ad, bd, id, acc);
+                                        acc = true;
+                                    }
+                                }
+                            }
+                            umma::commit(mbar);
+                        }
+                        wait_mma();
+                        CHAIN_PROF(4);
+                        // ---- epilogue: C -= dC (rows: TMEM lanes), store tile rows + slot rows ----
+                        {
+                            auto rows_out = [&](int row, const float (&v)[16]) {
+#pragma unroll
+                                for (int n = 0; n < CW; ++n) {
+                                    const float cn = fmaf(-v[n], wscale[n], Cs[(size_t)n * VP + row]);
+                                    Cs[(size_t)n * VP + row] = cn;
+                                    if (n < ncb && row < h && !(leaf && row < hr0)) A[(cb0 + n) * lda + s + row] = cn;
+                                }
+                            };
+                            float v[16];
+                            umma::tmem_ld16(tmem + ((uint32_t)(32 * warp) << 16) + Cfg::TM_D1, v);
+                            rows_out(32 * warp + lane, v);
+                            if constexpr (Cfg::B > 128) {
+                                umma::tmem_ld16(tmem + ((uint32_t)(32 * warp) << 16) + Cfg::TM_D2, v);
+                                if constexpr (Cfg::B - 128 >= 128) {
+                                    rows_out(128 + 32 * warp + lane, v);
+                                } else {
+                                    if (lane < 16) rows_out(128 + 16 * warp + lane, v);
+                                }
+                            }
+                            if (!leaf)
+                                for (int e = tid; e < CW * 32; e += Cfg::NT) {
+                                    const int n = e >> 5, i = e & 31;
+                                    if (n < ncb && i < wp) A[(cb0 + n) * lda + slotp + i] = Csl[n * 32 + i];
+                                }
+                        }
+                        umma::fence_before_sync();
+                        __syncthreads();
+                        CHAIN_PROF(8);
+                    }
+                } else {
+                __syncthreads();
+                    chain_gemm_gram<Cfg>(Vs, Gs);  // G = V^T V (tile part)
                     __syncthreads();
-                    CHAIN_PROF(4);
-                    chain_store<Cfg>(Cs, Csl, A, lda, cb0, ncb, s, h, slotp, wp, leaf, hr0);
-                    if (ib + 1 < nchunk) __syncthreads();
+                    if (tid < 32) chain_build_t(Gs, taus, wp, Ts, Tws + (t * g.npan + p) * (kPW * kPW), HS);
+    
+                    if (nchunk > 0) {
+                        int64_t cb;
+                        const int n0c = chunk_cols(cid(0), &cb);
+                        chain_stage<Cfg>(sm + Cfg::OFF_C, sm + Cfg::OFF_CS, A, lda, cb, n0c, s, h, slotp, wp, leaf, hr0);
+                    }
+                    for (int ib = 0; ib < nchunk; ++ib) {
+                        int64_t cb0;
+                        const int ncb = chunk_cols(cid(ib), &cb0);
+                        float* Cs = sm + Cfg::OFF_C + (ib & 1) * CW * VP;
+                        float* Csl = sm + Cfg::OFF_CS + (ib & 1) * CW * 32;
+                        if (ib + 1 < nchunk) {  // prefetch the next chunk into the other buffer
+                            int64_t cb1;
+                            const int n1c = chunk_cols(cid(ib + 1), &cb1);
+                            chain_stage<Cfg>(sm + Cfg::OFF_C + ((ib + 1) & 1) * CW * VP,
+                                             sm + Cfg::OFF_CS + ((ib + 1) & 1) * CW * 32, A, lda, cb1, n1c, s, h, slotp, wp,
+                                             leaf, hr0);
+                            asm volatile("cp.async.wait_group 1;" ::: "memory");
+                        } else {
+                            asm volatile("cp.async.wait_group 0;" ::: "memory");
+                        }
+                        __syncthreads();
+                        CHAIN_PROF(3);
+                        chain_gemm_vtc<Cfg>(Vs, Cs, Csl, !leaf, sm + Cfg::OFF_W);
+                        __syncthreads();
+                        chain_gemm_tw<Cfg>(Ts, sm + Cfg::OFF_W, sm + Cfg::OFF_W2);
+                        __syncthreads();
+                        if (!leaf)  // slot rows: C_slot -= W2 (V's head part is the identity)
+                            for (int e = tid; e < CW * 32; e += Cfg::NT) {
+                                const int cc = e >> 5, i = e & 31;
+                                Csl[cc * 32 + i] -= sm[Cfg::OFF_W2 + i * Cfg::WS + cc];
+                            }
+                        chain_gemm_update<Cfg>(Vs, Cs, sm + Cfg::OFF_W2);
+                        __syncthreads();
+                        CHAIN_PROF(4);
+                        chain_store<Cfg>(Cs, Csl, A, lda, cb0, ncb, s, h, slotp, wp, leaf, hr0);
+                        if (ib + 1 < nchunk) __syncthreads();
+                    }
                 }
                 if (nchunk > 0) {
                     // the next panel's columns (chunks 0 and 1, the last two
@@ -681,7 +1024,12 @@ tsqr_chain_kernel(Geom g, float* __restrict__ A, float* __restrict__ Tws, int* _
         CHAIN_PROF(5);
     }
     if (prof && threadIdx.x == 0)
-        for (int k = 0; k < 6; ++k) atomicAdd(prof + k, pacc[k]);
+        for (int k = 0; k < 10; ++k) atomicAdd(prof + k, pacc[k]);
+    if constexpr (TC) {  // every MMA has completed (each chunk waited on its commit)
+        umma::fence_before_sync();
+        __syncthreads();
+        if (threadIdx.x < 32) umma::tmem_free<128>(s_tmem);
+    }
 #undef CHAIN_PROF
 }
 
