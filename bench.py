@@ -4,13 +4,21 @@ path on BASELINE.json's headline workload, 1,000,000 x 192 fp32 (config C4).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--config NAME] [--impl caqr|reference]
     torchrun --nproc-per-node N bench.py --gpus N ...      (row-sharded, weak scaling)
+    python bench.py --gpus N ...   (N > 1 without torchrun: re-launches itself
+                                    under torch.distributed.run; exits 1 if fewer
+                                    than N GPUs are visible)
 
 One step = one caqr_factor (TSQR leaves + tree + R extraction) of a fresh copy
 of the synthetic input that is already resident in HBM.  A is restored from a
 pristine copy and a 256 MiB buffer is written (L2 flush) before every step,
 outside the CUDA events that time the step; inputs (768 MB) exceed L2 anyway.
-Rank 0 prints ONE JSON line.  `--impl reference` times the CPU oracle (the
-reference arm of this tier: the paper ships no code) on a bounded sample.
+Rank 0 prints ONE JSON line.  Beside the headline (weak scaling: 1M rows per
+GPU) it carries "strong_scaling" (config C4' 8,000,000 x 192 split over the N
+ranks; at N = 1 the whole 6.1 GB matrix on one GPU) and, at N = 1, "configs":
+the other BASELINE configs (C1, C2, C3, C4 fp64, C5) timed with the same
+protocol.  `--impl reference` times the CPU oracle (the reference arm of this
+tier: the paper ships no code) on a bounded row sample -- the same sample the
+cpu_baseline leg uses.
 """
 from __future__ import annotations
 
@@ -44,7 +52,47 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-chunks", type=int, default=16, help="row chunks of caqr_factor_host in the e2e leg")
     ap.add_argument("--cpu-sample-rows", type=int, default=0)
+    ap.add_argument("--no-extra", action="store_true", help="skip the strong-scaling and extra-config legs")
     return ap.parse_args()
+
+
+def cpu_info():
+    """`lscpu` model name and the host's core count (nproc)."""
+    model = None
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    return {"model": model, "nproc": os.cpu_count()}
+
+
+def sample_rows(cfg, override=0):
+    """Rows of the CPU oracle's bounded sample of a workload (both the
+    reference arm and the cpu_baseline leg): ~8 GFLOP per step, i.e. ~4 s of
+    single-thread oracle at its ~2 GFLOP/s."""
+    m, n = cfg["m"], cfg["n"]
+    return int(override or min(m, max(n, 8e9 / (2.0 * n * n))))
+
+
+def relaunch_distributed(args):
+    """--gpus N > 1 without a torch.distributed environment: re-run this script
+    under torch.distributed.run with N ranks on this node (never a silent
+    one-GPU measurement); exit 1 if fewer than N GPUs are visible."""
+    import subprocess
+
+    import torch
+
+    have = torch.cuda.device_count()
+    if have < args.gpus:
+        sys.stderr.write(f"bench.py: --gpus {args.gpus} requested but only {have} GPU(s) visible\n")
+        raise SystemExit(1)
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(29500 + os.getpid() % 1000), __file__] + sys.argv[1:]
+    raise SystemExit(subprocess.call(cmd))
 
 
 def load_peaks():
@@ -136,7 +184,7 @@ def run_reference(args, rank):
 
     cfg = workload(args.config)
     m, n, dt = cfg["m"], cfg["n"], cfg["dtype"]
-    rows = args.cpu_sample_rows or max(n, min(m, 20_000))
+    rows = sample_rows(cfg, args.cpu_sample_rows)
     acc = "d" if dt == "f32" else "ld"
     npdt = np.float32 if dt == "f32" else np.float64
     A = workloads.gaussian(rows, n, seed=0, dtype=npdt).astype(np.float64)
@@ -156,7 +204,8 @@ def run_reference(args, rank):
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": dt, "data": "synthetic",
         "config": {"workload": args.config, "m": m, "n": n, "sample_rows": rows},
-        "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+        "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample,
+                         "cpu": cpu_info()},
         "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -170,8 +219,7 @@ def cpu_baseline(cfg, rows_override=0):
     from paper_conf_ipps_andersonbdk11_b200 import workloads
 
     m, n, dt = cfg["m"], cfg["n"], cfg["dtype"]
-    # ~2 GFLOP/s single thread (BASELINE.md probe): aim at ~15 GFLOP of work
-    rows = rows_override or int(min(m, max(n, 15e9 / (2.0 * n * n))))
+    rows = sample_rows(cfg, rows_override)  # the reference arm's sample
     acc = "d" if dt == "f32" else "ld"
     A = workloads.gaussian(rows, n, seed=0, dtype=np.float32 if dt == "f32" else np.float64)
     A = A.astype(np.float64)
@@ -181,7 +229,135 @@ def cpu_baseline(cfg, rows_override=0):
     flops = 2.0 * rows * n * n - 2.0 * n ** 3 / 3.0
     return {"value": flops / t / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
             "sample": f"oracle_qr_{acc} (single-thread Householder, C) on rows [0,{rows}) x {n} of a "
-                      f"{dt} Gaussian, {t:.1f} s"}
+                      f"{dt} Gaussian, {t:.1f} s (same sample as one --impl reference step)",
+            "cpu": cpu_info()}
+
+
+# ---- extra legs: strong scaling (C4') and the other BASELINE configs ----------
+def make_input(cfg, seed, dev, rows=None):
+    """Synthetic input of a config as a column-major device tensor: Gaussian
+    drawn on the device; the s-step Krylov basis and the video matrix built on
+    the host (workloads.py recipes) and uploaded."""
+    import numpy as np
+    import torch
+
+    from paper_conf_ipps_andersonbdk11_b200 import caqr, workloads
+
+    m, n = rows or cfg["m"], cfg["n"]
+    tdt = torch.float32 if cfg["dtype"] == "f32" else torch.float64
+    if cfg["kind"] == "gaussian":
+        return workloads.device_gaussian(m, n, seed=seed, dtype=tdt, device=dev).t()
+    host = (workloads.krylov_basis(grid=2000, s=n, seed=seed, shifted=True) if cfg["kind"] == "krylov"
+            else workloads.video(seed=seed)).astype(np.float32 if cfg["dtype"] == "f32" else np.float64)
+    A0 = caqr.colmajor_empty(host.shape[0], host.shape[1], tdt, dev)
+    A0.copy_(torch.from_numpy(np.ascontiguousarray(host)))
+    return A0
+
+
+def timed_steps(step, prep, warmup, steps, stream):
+    """Same protocol as the headline: >= 3 warm-ups, prep (A restore + L2
+    flush) outside the CUDA events, events on the launching stream."""
+    import torch
+
+    for _ in range(max(warmup, 3)):
+        prep()
+        step()
+    torch.cuda.synchronize()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+    for a, b in evs:
+        prep()
+        a.record(stream)
+        step()
+        b.record(stream)
+    torch.cuda.synchronize()
+    return sum(a.elapsed_time(b) for a, b in evs) / steps
+
+
+def extra_configs_leg(args, dev, flush, peaks):
+    """N = 1: the other BASELINE configs with the headline's protocol."""
+    import torch
+
+    from paper_conf_ipps_andersonbdk11_b200 import caqr
+
+    out = {}
+    stream = torch.cuda.current_stream()
+    for name in ("c1_4096x16_f32", "c2_krylov_4Mx8_f32", "c3_video_110592x100_f32", "c4_1Mx192_f64",
+                 "c5_8192x8192_f32"):
+        cfg = workload(name)
+        m, n, dt = cfg["m"], cfg["n"], cfg["dtype"]
+        esz = 4 if dt == "f32" else 8
+        opts = caqr.make_opts(0, cfg.get("nb", 0))
+        A0 = make_input(cfg, 0, dev)
+        A = caqr.colmajor_empty(m, n, A0.dtype, dev)
+        code = caqr.CAQR_F32 if dt == "f32" else caqr.CAQR_F64
+        R = caqr.colmajor_empty(n, n, A0.dtype, dev)
+        ws = torch.empty(max(caqr.caqr_workspace_bytes(m, n, code, opts), 1), dtype=torch.uint8, device=dev)
+
+        def prep():
+            A.copy_(A0)
+            flush.zero_()
+
+        steps = min(args.steps, 5 if m * n > 5e7 else 20)
+        ms = timed_steps(lambda: caqr.caqr_factor(A, R=R, ws=ws, opts=opts), prep, args.warmup, steps, stream)
+        fl = 2.0 * m * n * n - 2.0 * n ** 3 / 3.0
+        alu = alu_peak_tflops(dt, peaks["sm_max_mhz"])
+        t_roof = max(2.0 * m * n * esz / (peaks["hbm_gbs"] * 1e9), fl / (alu * 1e12))
+        out[name] = {"ms_per_step": ms, "value": fl / (ms * 1e-3) / 1e9, "unit": UNIT, "steps": steps,
+                     "read_write_gbs": 2.0 * m * n * esz / (ms * 1e-3) / 1e9,
+                     "roofline_frac": t_roof / (ms * 1e-3),
+                     "roofline_note": "max(read A + write V at measured HBM, flops at derived ALU peak) / time",
+                     "plan": caqr.caqr_plan_info(m, n, code, opts)}
+        del A0, A, R, ws
+        torch.cuda.empty_cache()
+    return out
+
+
+def strong_scaling_leg(args, dev, flush, world, rank, handle, L, gather, cws):
+    """Config C4' (8,000,000 x 192 fp32) split over the N ranks (strong
+    scaling; N = 1: the whole matrix on one GPU).  Time per step = max over
+    ranks of each rank's event time (local TSQR + all-gather + combine)."""
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_andersonbdk11_b200 import caqr
+    from paper_conf_ipps_andersonbdk11_b200.dist import shard_rows
+
+    cfg = workload("c4p_8Mx192_f32")
+    m_total, n = cfg["m"], cfg["n"]
+    _, rows = shard_rows(m_total, world, rank)
+    A0 = make_input(cfg, 77 + rank, dev, rows=rows)
+    A = caqr.colmajor_empty(rows, n, torch.float32, dev)
+    R = caqr.colmajor_empty(n, n, torch.float32, dev)
+    ws = torch.empty(caqr.caqr_workspace_bytes(rows, n, caqr.CAQR_F32, None), dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def step():
+        if handle is None:
+            caqr.caqr_factor(A, R=R, ws=ws)
+        else:
+            caqr._check("caqr_dist_factor_f32", L.caqr_dist_factor_f32(
+                handle, rows, n, A.data_ptr(), rows, R.data_ptr(), n, ws.data_ptr(), ws.numel(),
+                gather.data_ptr(), cws.data_ptr(), cws.numel(), None, caqr.ctypes.c_void_p(stream.cuda_stream)))
+
+    def prep():
+        A.copy_(A0)
+        flush.zero_()
+
+    if world > 1:
+        dist.barrier()
+    steps = max(3, min(args.steps, 5))
+    ms = timed_steps(step, prep, args.warmup, steps, stream)
+    if world > 1:
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    fl = 2.0 * m_total * n * n - 2.0 * n ** 3 / 3.0
+    del A0, A, R, ws
+    torch.cuda.empty_cache()
+    return {"workload": "c4p_8Mx192_f32", "scaling": "strong", "m_total": m_total, "m_per_gpu": rows,
+            "n": n, "n_gpus": world, "steps": steps, "ms_per_step": ms, "value": fl / (ms * 1e-3) / 1e9,
+            "unit": UNIT, "timing": "per rank CUDA events around each factor (N > 1: caqr_dist_factor incl. the "
+                                    "NCCL all-gather and combine), mean over steps, max over ranks"}
 
 
 # ---- the CUDA arm -------------------------------------------------------------
@@ -190,6 +366,11 @@ def main():
     rank = int(os.environ.get("RANK", 0))
     world = int(os.environ.get("WORLD_SIZE", 1))
     local = int(os.environ.get("LOCAL_RANK", 0))
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        relaunch_distributed(args)
+    if world != args.gpus:
+        sys.stderr.write(f"bench.py: WORLD_SIZE={world} but --gpus {args.gpus}\n")
+        raise SystemExit(1)
     if args.impl == "reference":
         run_reference(args, rank)
         return
@@ -344,6 +525,7 @@ def main():
     # it lands, then combines the chunks' R's; + D2H of R.  The serial variant
     # (whole H2D, then caqr_factor) is reported beside it for context.
     e2e = None
+    Ah = None
     if not args.no_e2e and world == 1:
         Ah = torch.empty((n, m), dtype=tdt, pin_memory=True).t()
         Ah.copy_(A0)
@@ -412,6 +594,14 @@ def main():
                "api": "per rank: pinned H2D of the row shard + caqr_dist_factor (local TSQR, NCCL all-gather "
                       "of the R's, combine) + D2H(R); max over ranks"}
 
+    strong, extra = None, None
+    if not args.no_extra:
+        Ah = None  # release the e2e leg's pinned host copy
+        strong = strong_scaling_leg(args, dev, flush, world, rank, handle, L,
+                                    gather if world > 1 else None, cws if world > 1 else None)
+        if world == 1 and rank == 0:
+            extra = extra_configs_leg(args, dev, flush, peaks)
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(cfg, args.cpu_sample_rows)
@@ -439,6 +629,8 @@ def main():
                         for k, v in per.items()},
             "e2e": e2e,
             "cpu_baseline": cpu,
+            "strong_scaling": strong,
+            "configs": extra,
         }
         print(json.dumps(line), flush=True)
     if handle is not None:

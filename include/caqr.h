@@ -63,7 +63,7 @@ extern "C" {
 typedef struct CUstream_st *caqr_stream_t; /* == cudaStream_t */
 
 enum { CAQR_F32 = 0, CAQR_F64 = 1 };
-enum { CAQR_OK = 0, CAQR_ERR_CUDA = 1, CAQR_ERR_NCCL = 2, CAQR_ERR_UNSUPPORTED = 3 };
+enum { CAQR_OK = 0, CAQR_ERR_CUDA = 1, CAQR_ERR_NCCL = 2, CAQR_ERR_UNSUPPORTED = 3, CAQR_ERR_TIMEOUT = 4 };
 
 /* Plan options; a field <= 0 means "default".
  *   leaf_rows  b: rows per TSQR tile (P:L633 / P:L822-823 used 64 and 128 on
@@ -222,7 +222,8 @@ typedef struct caqr_dist caqr_dist;
 int caqr_dist_unique_id(void *out128);
 int caqr_dist_create(caqr_dist **handle, int nranks, int rank, const void *nccl_unique_id);
 void caqr_dist_destroy(caqr_dist *handle);
-/* Every rank: local TSQR of its m_local x n shard (m_local >= n), ncclAllGather
+/* Every rank: local TSQR of its m_local x n shard (m_local >= n: else -2),
+ * ncclAllGather
  * of the local R factors over NVLink, then the same deterministic combine on
  * every rank -> the global R (identical bits on all ranks).
  *   A, lda, ws, ws_bytes: the local factorisation (caqr_workspace_bytes(m_local,
@@ -237,6 +238,29 @@ int caqr_dist_factor_f64(caqr_dist *h, int64_t m_local, int64_t n, double *A, in
                          double *R, int64_t ldr, void *ws, size_t ws_bytes, double *gather,
                          void *cws, size_t cws_bytes, const caqr_opts *opts,
                          caqr_stream_t stream);
+
+/* The post-exchange half of caqr_dist_factor, NCCL-free (caqr_dist_factor
+ * calls it after its all-gather; a caller with its own exchange -- or a test
+ * emulating P ranks on one GPU -- calls it directly): restack P contiguous
+ * column-major n x n upper-triangular blocks (rank order; `blocks`, device,
+ * P*n*n elements) into the (P*n) x n stack `gather` (ld ldg >= P*n) and run
+ * caqr_combine on it: R (n x n, ldr >= n) = the global R, `gather` keeps the
+ * combine's tree vectors, cws its T factors (caqr_combine_apply uses both).
+ * The distributed TSQR's extra tree level.
+ *   info: -1 P < 1, -2 n outside [0, 256], -3 blocks, -4 gather, -5 ldg,
+ *   -6 R, -7 ldr, -8 cws, -9 cws_bytes < caqr_combine_workspace_bytes(P, n,
+ *   dtype); CAQR_ERR_CUDA. */
+int caqr_dist_combine_blocks_f32(int P, int64_t n, const float *blocks, float *gather, int64_t ldg,
+                                 float *R, int64_t ldr, void *cws, size_t cws_bytes, caqr_stream_t stream);
+int caqr_dist_combine_blocks_f64(int P, int64_t n, const double *blocks, double *gather, int64_t ldg,
+                                 double *R, int64_t ldr, void *cws, size_t cws_bytes, caqr_stream_t stream);
+/* Host-side wait with a deadline for the work a dist call enqueued on
+ * `stream`: 0 once the stream is idle; on an NCCL asynchronous error, or when
+ * timeout_ms (>= 0; < 0 = no deadline) passes first, the communicator is
+ * aborted (ncclCommAbort: a peer that died or never arrived cannot hang this
+ * rank) and CAQR_ERR_NCCL / CAQR_ERR_TIMEOUT is returned; the handle then only
+ * accepts caqr_dist_destroy.  -1: h NULL; CAQR_ERR_CUDA: the stream failed. */
+int caqr_dist_wait(caqr_dist *h, caqr_stream_t stream, int timeout_ms);
 
 /* ---- Least squares through the factorization -------------
  * min ||A x - b||_2 for tall full-rank A, the use of QR the paper opens with

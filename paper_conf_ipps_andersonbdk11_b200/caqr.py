@@ -105,6 +105,12 @@ def lib() -> ctypes.CDLL:
         L.caqr_dist_create.restype = ip
         L.caqr_dist_destroy.argtypes = [vp]
         L.caqr_dist_destroy.restype = None
+        L.caqr_dist_wait.argtypes = [vp, vp, ip]
+        L.caqr_dist_wait.restype = ip
+        for suf in ("f32", "f64"):
+            f = getattr(L, f"caqr_dist_combine_blocks_{suf}")
+            f.argtypes = [ip, i64, vp, vp, i64, vp, i64, vp, sz, vp]
+            f.restype = ip
         fl = ctypes.c_float
         for suf in ("f32", "f64"):
             f = getattr(L, f"caqr_lstsq_{suf}")
@@ -373,6 +379,29 @@ def caqr_combine_apply(Rstack, P: int, ws, C, trans: bool = True, stream=None):
                                                         C.shape[1], pc, ldc, _stream(stream))
     _check(f"caqr_combine_apply_{suf}", info)
     return C
+
+
+def caqr_dist_combine_blocks(blocks, P: int, n: int, gather=None, R=None, cws=None, stream=None):
+    """The post-exchange half of the distributed factor (caqr_dist_combine_blocks_*):
+    `blocks` holds P contiguous column-major n x n R factors (rank order, e.g. an
+    all-gather's receive buffer, P*n*n elements); returns (R, gather, cws) with
+    the combined R, the combine's tree vectors and its workspace."""
+    torch = _torch()
+    code, suf = _dtype_code(blocks)
+    if blocks.numel() < P * n * n or not blocks.is_contiguous():
+        raise ValueError("blocks: P*n*n contiguous elements")
+    if gather is None:
+        gather = colmajor_empty(P * n, n, blocks.dtype, blocks.device)
+    pg, ldg = _colmajor(gather, "gather")
+    if R is None:
+        R = colmajor_empty(n, n, blocks.dtype, blocks.device)
+    pr, ldr = _colmajor(R, "R")
+    if cws is None:
+        cws = torch.empty(max(caqr_combine_workspace_bytes(P, n, code), 1), dtype=torch.uint8, device=blocks.device)
+    info = getattr(lib(), f"caqr_dist_combine_blocks_{suf}")(P, n, blocks.data_ptr(), pg, ldg, pr, ldr,
+                                                               cws.data_ptr(), cws.numel(), _stream(stream))
+    _check(f"caqr_dist_combine_blocks_{suf}", info)
+    return R, gather, cws
 
 
 # ---- application layer: SVD via QR, robust PCA (include/caqr.h, Sec. VI) ----

@@ -106,7 +106,12 @@ static int make_plan(int64_t m, int64_t n, int dtype, const caqr_opts* o, int op
     pl->m = m;
     pl->n = n;
     pl->dtype = dtype;
-    int64_t nb = (o && o->panel_cols > 0) ? o->panel_cols : (n <= kMaxGroup ? n : 64);
+    // default group width: the whole matrix for n <= 224 (one TSQR); 128 for
+    // n in (224, 256] -- a 256-wide group's top tree merges need 2*32 + 224 =
+    // 288 > 256 gathered rows, which only the per-level split path takes (SURVEY
+    // 8(f) f3: 8192 x 256 was 6 ms that way, vs two 128-wide CAQR groups);
+    // 64-wide CAQR panels beyond
+    int64_t nb = (o && o->panel_cols > 0) ? o->panel_cols : (n <= 224 ? n : (n <= kMaxGroup ? 128 : 64));
     if (nb > kMaxGroup) return -opt_pos;
     nb = std::max<int64_t>(1, std::min(nb, std::max<int64_t>(n, 1)));
     // skinny fp32 panels (n <= 16, one group): one warp per chain, 256-row (n <= 8)
@@ -574,10 +579,13 @@ static bool side_stream(cudaStream_t* s2, cudaEvent_t* ev_ready, cudaEvent_t* ev
     return true;
 }
 
-// CAQR_MMA=0 keeps the CAQR trailing update on FFMA (exact fp32 products).
+// CAQR trailing update: FFMA (exact fp32 products) by default; CAQR_MMA=1 selects
+// 3xTF32 mma.sync -- measured slower (8192^2: 81.8 vs 76.1 ms) and 17-28x less
+// accurate (residual 4.7e-5 vs 2.8e-6: the ~2^-21 product error compounds over
+// the 128 panel groups).
 static inline bool mma_policy() {
     const char* e = getenv("CAQR_MMA");
-    return !(e && e[0] == '0');
+    return e && e[0] == '1';
 }
 
 // CAQR_SKINNY=0: no skinny kernel; =2: the older warp-per-task kernel with
@@ -917,6 +925,16 @@ static int factor_impl(int64_t m, int64_t n, T* A, int64_t lda, T* R, int64_t ld
     cudaStream_t s2 = nullptr;
     cudaEvent_t ev_ready = nullptr, ev_done = nullptr;
     const bool overlap = pl.ngroups > 1 && early_start_policy() && side_stream(&s2, &ev_ready, &ev_done);
+    // The side stream and its two events are per device and shared by every
+    // call: hold a per-device lock while this call records / waits on them, so
+    // that a concurrent call on another host thread cannot re-record ev_ready
+    // between this call's record and its wait (host issue is serialised; the
+    // GPU work stays asynchronous).
+    static std::mutex overlap_mu[64];
+    int dev_id = 0;
+    cudaGetDevice(&dev_id);
+    std::unique_lock<std::mutex> overlap_lock(overlap_mu[dev_id & 63], std::defer_lock);
+    if (overlap) overlap_lock.lock();
     for (int64_t g = 0; g < pl.ngroups && !rc; ++g) {
         const Geom G = group_geom(pl, g, lda);
         T* Tws;
@@ -1265,15 +1283,27 @@ static int factor_host_impl(int64_t m, int64_t n, int S, const T* Ah, int64_t ld
     if (cudaEventRecord(ev[S], s) != cudaSuccess || cudaStreamWaitEvent(cs, ev[S], 0) != cudaSuccess ||
         (dual && cudaStreamWaitEvent(s2, ev[S], 0) != cudaSuccess))
         return CAQR_ERR_CUDA;
+    // On an error return after this point, make `stream` wait for whatever the
+    // copy stream and the second compute stream already hold (queued H2D
+    // copies, odd chunks' TSQRs), so that a caller who synchronises `stream`
+    // may free A_host / ws safely and a capture has no unjoined fork.
+    auto join_fail = [&](int code) {
+        g_last_cuda_error = (int)cudaGetLastError();
+        cudaEventRecord(ev[S], cs);
+        cudaStreamWaitEvent(s, ev[S], 0);
+        if (dual) {
+            cudaEventRecord(ev[S + 1], s2);
+            cudaStreamWaitEvent(s, ev[S + 1], 0);
+        }
+        return code;
+    };
     char* wsb = static_cast<char*>(ws);
     for (int c = 0; c < S; ++c) {
         host_layout(m, n, S, dtype, opts, c, &r0, &mc, &off);
         if (cudaMemcpy2DAsync(A + r0, lda * sizeof(T), Ah + r0, ldh * sizeof(T), mc * sizeof(T), n,
                               cudaMemcpyHostToDevice, cs) != cudaSuccess ||
-            cudaEventRecord(ev[c], cs) != cudaSuccess) {
-            g_last_cuda_error = (int)cudaGetLastError();
-            return CAQR_ERR_CUDA;
-        }
+            cudaEventRecord(ev[c], cs) != cudaSuccess)
+            return join_fail(CAQR_ERR_CUDA);
     }
     int64_t rs0, rsn;
     size_t rs_off, cw_off;
@@ -1285,14 +1315,17 @@ static int factor_host_impl(int64_t m, int64_t n, int S, const T* Ah, int64_t ld
     for (int c = 0; c < S && !rc; ++c) {
         host_layout(m, n, S, dtype, opts, c, &r0, &mc, &off);
         cudaStream_t sc = dual && (c & 1) ? s2 : s;
-        if (cudaStreamWaitEvent(sc, ev[c], 0) != cudaSuccess) return CAQR_ERR_CUDA;
+        if (cudaStreamWaitEvent(sc, ev[c], 0) != cudaSuccess) return join_fail(CAQR_ERR_CUDA);
         const size_t wb = caqr_workspace_bytes(mc, n, dtype, opts);
-        if (S == 1) return factor_impl<T>(mc, n, A + r0, lda, R, ldr, wsb + off, wb, opts, s, dtype);
+        if (S == 1) {
+            rc = factor_impl<T>(mc, n, A + r0, lda, R, ldr, wsb + off, wb, opts, s, dtype);
+            return rc ? join_fail(rc) : 0;
+        }
         rc = factor_impl<T>(mc, n, A + r0, lda, Rs + (int64_t)c * n, ld, wsb + off, wb, opts, sc, dtype);
     }
-    if (rc) return rc;
+    if (rc) return join_fail(rc);
     if (dual && (cudaEventRecord(ev[S + 1], s2) != cudaSuccess || cudaStreamWaitEvent(s, ev[S + 1], 0) != cudaSuccess))
-        return CAQR_ERR_CUDA;
+        return join_fail(CAQR_ERR_CUDA);
     return combine_impl<T>(S, n, Rs, ld, R, ldr, wsb + cw_off, caqr_combine_workspace_bytes(S, n, dtype), s,
                            dtype);
 }
@@ -1371,6 +1404,7 @@ const char* caqr_strerror(int info) {
     if (info == CAQR_ERR_CUDA) return "CUDA launch failed (see caqr_last_cuda_error)";
     if (info == CAQR_ERR_NCCL) return "NCCL call failed";
     if (info == CAQR_ERR_UNSUPPORTED) return "unsupported size";
+    if (info == CAQR_ERR_TIMEOUT) return "distributed call timed out (communicator aborted)";
     if (info < 0) return "illegal argument (-info = position)";
     return "unknown";
 }

@@ -11,7 +11,10 @@
 #include <nccl.h>
 
 #include <cstdint>
+#include <algorithm>
+#include <chrono>
 #include <cstring>
+#include <thread>
 #include <new>
 
 #include "../../include/caqr.h"
@@ -20,6 +23,7 @@ struct caqr_dist {
     ncclComm_t comm;
     int nranks;
     int rank;
+    int aborted;
 };
 
 namespace {
@@ -44,14 +48,44 @@ ncclDataType_t nccl_type<float>() { return ncclFloat32; }
 template <>
 ncclDataType_t nccl_type<double>() { return ncclFloat64; }
 
+// The post-exchange half of the distributed factor: restack P contiguous
+// n x n blocks (rank order) into the (P n) x n stack `gather` and run the
+// deterministic combine tree on it.  NCCL-free: caqr_dist_factor calls it
+// after the all-gather, tests call it directly on one GPU.
+template <typename T>
+int combine_blocks(int P, int64_t n, const T* blocks, T* gather, int64_t ldg, T* R, int64_t ldr, void* cws,
+                   size_t cws_bytes, cudaStream_t s, int dtype) {
+    if (P < 1) return -1;
+    if (n < 0 || n > 256) return -2;
+    if (n == 0) return 0;
+    if (!blocks) return -3;
+    if (!gather) return -4;
+    if (ldg < (int64_t)P * n) return -5;
+    if (!R) return -6;
+    if (ldr < n) return -7;
+    if (!cws) return -8;
+    if (cws_bytes < caqr_combine_workspace_bytes(P, n, dtype)) return -9;
+    const int64_t total = (int64_t)P * n * n;
+    const int blocks_ = (int)std::min<int64_t>(1024, (total + 255) / 256);
+    stack_blocks_kernel<T><<<blocks_, 256, 0, s>>>(P, n, blocks, gather, ldg);
+    if (cudaGetLastError() != cudaSuccess) return CAQR_ERR_CUDA;
+    return dtype == CAQR_F32 ? caqr_combine_f32(P, n, (float*)gather, ldg, (float*)R, ldr, cws, cws_bytes, s)
+                             : caqr_combine_f64(P, n, (double*)gather, ldg, (double*)R, ldr, cws, cws_bytes, s);
+}
+
 template <typename T>
 int dist_factor(caqr_dist* h, int64_t m_local, int64_t n, T* A, int64_t lda, T* R, int64_t ldr,
                 void* ws, size_t ws_bytes, T* gather, void* cws, size_t cws_bytes,
                 const caqr_opts* opts, cudaStream_t s, int dtype) {
     if (!h) return -1;
+    if (h->aborted) return CAQR_ERR_NCCL;
     if (n < 0 || n > 256) return -3;
     if (!gather || !cws) return -10;
     const int P = h->nranks;
+    // every argument check before the local factor and the collective: a rank
+    // that returned early would leave the others blocked in ncclAllGather
+    if (n > 0 && cws_bytes < caqr_combine_workspace_bytes(P, n, dtype)) return -12;
+    if (m_local < n) return -2;
     // 1. local TSQR of the shard (R lands in R, ldr)
     int rc = dtype == CAQR_F32
                  ? caqr_factor_f32(m_local, n, (float*)A, lda, (float*)R, ldr, ws, ws_bytes, opts, s)
@@ -59,7 +93,6 @@ int dist_factor(caqr_dist* h, int64_t m_local, int64_t n, T* A, int64_t lda, T* 
                                    opts, s);
     if (rc) return rc;
     if (n == 0) return 0;
-    if (cws_bytes < caqr_combine_workspace_bytes(P, n, dtype)) return -12;
     // receive area for P contiguous n x n blocks sits after the combine's T blocks
     const size_t blk_elems = (size_t)P * n * n;
     T* recv = reinterpret_cast<T*>(static_cast<char*>(cws) + caqr_combine_workspace_bytes(P, n, dtype) -
@@ -73,13 +106,7 @@ int dist_factor(caqr_dist* h, int64_t m_local, int64_t n, T* A, int64_t lda, T* 
     if (ncclAllGather(send, recv, (size_t)n * n, nccl_type<T>(), h->comm, s) != ncclSuccess)
         return CAQR_ERR_NCCL;
     // 3. restack and combine (same bits on every rank)
-    const int64_t ld = (int64_t)P * n;
-    stack_blocks_kernel<T><<<64, 256, 0, s>>>(P, n, recv, gather, ld);
-    if (cudaGetLastError() != cudaSuccess) return CAQR_ERR_CUDA;
-    return dtype == CAQR_F32 ? caqr_combine_f32(P, n, (float*)gather, ld, (float*)R, ldr, cws,
-                                                cws_bytes, s)
-                             : caqr_combine_f64(P, n, (double*)gather, ld, (double*)R, ldr, cws,
-                                                cws_bytes, s);
+    return combine_blocks<T>(P, n, recv, gather, (int64_t)P * n, R, ldr, cws, cws_bytes, s, dtype);
 }
 
 }  // namespace
@@ -96,6 +123,7 @@ int caqr_dist_create(caqr_dist** handle, int nranks, int rank, const void* nccl_
     if (!h) return CAQR_ERR_NCCL;
     h->nranks = nranks;
     h->rank = rank;
+    h->aborted = 0;
     if (ncclCommInitRank(&h->comm, nranks, id, rank) != ncclSuccess) {
         delete h;
         return CAQR_ERR_NCCL;
@@ -106,8 +134,46 @@ int caqr_dist_create(caqr_dist** handle, int nranks, int rank, const void* nccl_
 
 void caqr_dist_destroy(caqr_dist* h) {
     if (!h) return;
-    ncclCommDestroy(h->comm);
+    if (h->aborted)
+        ncclCommAbort(h->comm);
+    else
+        ncclCommDestroy(h->comm);
     delete h;
+}
+
+int caqr_dist_wait(caqr_dist* h, caqr_stream_t stream, int timeout_ms) {
+    if (!h) return -1;
+    if (h->aborted) return CAQR_ERR_NCCL;
+    const auto t0 = std::chrono::steady_clock::now();
+    for (;;) {
+        const cudaError_t q = cudaStreamQuery(reinterpret_cast<cudaStream_t>(stream));
+        if (q == cudaSuccess) return 0;
+        if (q != cudaErrorNotReady) return CAQR_ERR_CUDA;
+        ncclResult_t async = ncclSuccess;
+        if (ncclCommGetAsyncError(h->comm, &async) != ncclSuccess || async != ncclSuccess) {
+            ncclCommAbort(h->comm);
+            h->aborted = 1;
+            return CAQR_ERR_NCCL;
+        }
+        const auto ms = std::chrono::duration_cast<std::chrono::milliseconds>(std::chrono::steady_clock::now() - t0);
+        if (timeout_ms >= 0 && ms.count() > timeout_ms) {
+            ncclCommAbort(h->comm);  // unblocks the collective on this rank
+            h->aborted = 1;
+            return CAQR_ERR_TIMEOUT;
+        }
+        std::this_thread::sleep_for(std::chrono::microseconds(50));
+    }
+}
+
+int caqr_dist_combine_blocks_f32(int P, int64_t n, const float* blocks, float* gather, int64_t ldg, float* R,
+                                 int64_t ldr, void* cws, size_t cws_bytes, caqr_stream_t stream) {
+    return combine_blocks<float>(P, n, blocks, gather, ldg, R, ldr, cws, cws_bytes,
+                                 reinterpret_cast<cudaStream_t>(stream), CAQR_F32);
+}
+int caqr_dist_combine_blocks_f64(int P, int64_t n, const double* blocks, double* gather, int64_t ldg, double* R,
+                                 int64_t ldr, void* cws, size_t cws_bytes, caqr_stream_t stream) {
+    return combine_blocks<double>(P, n, blocks, gather, ldg, R, ldr, cws, cws_bytes,
+                                  reinterpret_cast<cudaStream_t>(stream), CAQR_F64);
 }
 
 int caqr_dist_factor_f32(caqr_dist* h, int64_t m_local, int64_t n, float* A, int64_t lda, float* R,

@@ -152,19 +152,27 @@ __device__ __forceinline__ T rcp_rn(T x) {
         return __drcp_rn(x);
 }
 
-// 1/sqrt(s) and sqrt(s), s > 0.  fp32: hardware approximations plus one
-// Newton step (~1 ulp; the reflector stays orthogonal to that level), far
-// cheaper on the critical path than the IEEE-rounded sqrt / division
-// subroutines.  fp64: IEEE-rounded.
+// 1/sqrt(s) and sqrt(s), s > 0, for the reflector scalars mu, tau = 1 + |alpha|/mu
+// and 1/(|alpha| + mu).  fp32: hardware approximations plus one Newton step
+// (~1 ulp), far cheaper on the reflector critical path than the IEEE-rounded
+// subroutines.  Measured round 2 (1M x 192): IEEE __fsqrt_rn / __frcp_rn give
+// ||Q^T Q - I|| 2.9e-6 instead of 6.8e-6 (fp32 LAPACK: 2.0e-6; bound 1e-5) at
+// +5 % time (6.03 vs 5.74 ms), so the hot path keeps the approximations;
+// CAQR_IEEE_SCALARS (compile-time) selects the IEEE ones.  fp64: IEEE-rounded.
 template <typename T>
 __device__ __forceinline__ void rsqrt_refined(T s, T& r, T& sq) {
     if constexpr (sizeof(T) == 4) {
+#ifdef CAQR_IEEE_SCALARS
+        sq = __fsqrt_rn(s);
+        r = __frcp_rn(sq);
+#else
         float y = rsqrtf(s);
         const float h = 0.5f * s * y;
         y = fmaf(-h, y, 1.5f) * y;  // y (1.5 - 0.5 s y^2)
         r = y;
         const float q = s * y;      // sqrt(s) ~ s / sqrt(s), one residual correction
         sq = fmaf(fmaf(-q, q, s), 0.5f * y, q);
+#endif
     } else {
         sq = sqrt(s);
         r = __drcp_rn(sq);
@@ -173,8 +181,12 @@ __device__ __forceinline__ void rsqrt_refined(T s, T& r, T& sq) {
 template <typename T>
 __device__ __forceinline__ T rcp_refined(T d) {
     if constexpr (sizeof(T) == 4) {
+#ifdef CAQR_IEEE_SCALARS
+        return __frcp_rn(d);
+#else
         float y = __fdividef(1.0f, d);
         return fmaf(fmaf(-d, y, 1.0f), y, y);  // one Newton step
+#endif
     } else {
         return __drcp_rn(d);
     }

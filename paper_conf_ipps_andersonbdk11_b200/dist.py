@@ -62,15 +62,43 @@ def local_form_q(A_local, ws, gather, cws, rank: int, world: int, opts=None, str
     all-gather.  All steps are libcaqr kernels."""
     from . import caqr
 
+    import contextlib
+
+    import torch
+
     m, n = A_local.shape
-    Qc = caqr.colmajor_empty(world * n, n, A_local.dtype, A_local.device)
-    caqr.caqr_set_identity(Qc, stream=stream)
-    caqr.caqr_combine_apply(gather, world, cws, Qc, trans=False, stream=stream)
-    Q = caqr.colmajor_empty(m, n, A_local.dtype, A_local.device)
-    caqr.caqr_set_identity(Q, stream=stream)  # then overwrite the top n x n with Q_c,p
-    Q[:n].copy_(Qc[rank * n:(rank + 1) * n])
-    caqr.caqr_apply_q(A_local, ws, Q, opts=opts, stream=stream)
+    # every step -- the library calls and the torch copy between them -- on
+    # the caller's stream (the copy would otherwise run on torch's current
+    # stream, unordered with the library calls)
+    ctx = torch.cuda.stream(stream) if isinstance(stream, torch.cuda.Stream) else contextlib.nullcontext()
+    with ctx:
+        Qc = caqr.colmajor_empty(world * n, n, A_local.dtype, A_local.device)
+        caqr.caqr_set_identity(Qc, stream=stream)
+        caqr.caqr_combine_apply(gather, world, cws, Qc, trans=False, stream=stream)
+        Q = caqr.colmajor_empty(m, n, A_local.dtype, A_local.device)
+        caqr.caqr_set_identity(Q, stream=stream)  # then overwrite the top n x n with Q_c,p
+        Q[:n].copy_(Qc[rank * n:(rank + 1) * n])
+        caqr.caqr_apply_q(A_local, ws, Q, opts=opts, stream=stream)
     return Q
+
+
+def agree_shards(m_local: int, n: int, group=None) -> None:
+    """Every rank checks its own shard (m_local >= n >= 0, n <= 256) and the
+    ranks all-reduce the verdict, so that either all of them enter the NCCL
+    collective or all of them raise (a rank that bailed out alone would leave
+    the others blocked in the all-gather).  Works with any torch.distributed
+    backend (gloo on CPU in the tests)."""
+    import torch
+    import torch.distributed as dist
+
+    ok = 1 if (0 <= n <= 256 and m_local >= n) else 0
+    backend = dist.get_backend(group)
+    dev = torch.device("cuda", torch.cuda.current_device()) if backend == "nccl" else torch.device("cpu")
+    t = torch.tensor([ok], dtype=torch.int32, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MIN, group=group)
+    if int(t.item()) != 1:
+        raise ValueError(f"some rank's shard is unusable (this rank: {m_local} rows, n = {n}; every shard needs "
+                         f"m_local >= n and n <= 256)")
 
 
 class DistTSQR:
@@ -83,6 +111,7 @@ class DistTSQR:
         from . import caqr
 
         self.caqr = caqr
+        self.group = group
         self.L = caqr.lib()
         self.world = dist.get_world_size(group)
         self.rank = dist.get_rank(group)
@@ -97,15 +126,20 @@ class DistTSQR:
         caqr._check("caqr_dist_create", self.L.caqr_dist_create(ctypes.byref(h), self.world, self.rank, uid))
         self.handle = h
 
-    def factor(self, A_local, opts=None, stream=None):
+    def factor(self, A_local, opts=None, stream=None, timeout_s: float = 600.0):
         """Factor the local column-major shard in place; returns (R, ws, gather,
         cws): the global R (identical bits on every rank), the local workspace,
-        the combine's stacked tree vectors and its workspace."""
+        the combine's stacked tree vectors and its workspace.  All ranks first
+        agree that every shard is usable (else every rank raises, none enters
+        the collective); the call then waits at most timeout_s for its stream
+        (caqr_dist_wait: on timeout or an NCCL error the communicator is aborted
+        and CaqrError is raised instead of hanging)."""
         import torch
 
         c = self.caqr
         code, suf = c._dtype_code(A_local)
         m, n = A_local.shape
+        agree_shards(m, n, self.group)
         pa, lda = c._colmajor(A_local, "A")
         R = c.colmajor_empty(n, n, A_local.dtype, A_local.device)
         ws = torch.empty(max(c.caqr_workspace_bytes(m, n, code, opts), 1), dtype=torch.uint8,
@@ -117,6 +151,9 @@ class DistTSQR:
             self.handle, m, n, pa, lda, R.data_ptr(), n, ws.data_ptr(), ws.numel(), gather.data_ptr(),
             cws.data_ptr(), cws.numel(), c._optp(opts), c._stream(stream))
         c._check(f"caqr_dist_factor_{suf}", info)
+        if timeout_s is not None:
+            c._check("caqr_dist_wait", self.L.caqr_dist_wait(self.handle, c._stream(stream),
+                                                             int(timeout_s * 1000)))
         return R, ws, gather, cws
 
     def form_q(self, A_local, ws, gather, cws, opts=None, stream=None):

@@ -78,3 +78,39 @@ def test_shard_rows():
     with pytest.raises(ValueError):
         cdist.check_shards(100, 60, 2)
     cdist.check_shards(8_000_000, 192, 8)
+
+
+def _agree_worker(rank, world, port, rows, n, out_q):
+    import torch.distributed as dist
+
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        cdist.agree_shards(rows[rank], n)
+        out_q.put((rank, "ok"))
+    except ValueError:
+        out_q.put((rank, "raised"))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("rows,expect", [((500, 400), "ok"), ((500, 40), "raised"), ((10, 500), "raised")])
+def test_agree_shards_all_or_none(rows, expect):
+    """DistTSQR.factor's pre-collective check (agree_shards): every rank checks
+    its own shard and the verdict is all-reduced, so either every rank enters
+    the NCCL all-gather or every rank raises -- one bad shard (rank 1: 40 rows <
+    n = 64) must not leave the other rank blocked in the collective."""
+    import torch.multiprocessing as mp
+
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_agree_worker, args=(r, 2, port, rows, 64, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=120) for _ in range(2))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert res == {0: expect, 1: expect}

@@ -46,6 +46,25 @@ def gpu_qr(c, A, opts=None, want_q=True):
     return R.cpu().numpy().astype(np.float64), (None if Q is None else Q.cpu().numpy().astype(np.float64)), Ad, ws
 
 
+def oracle_f_orth(A64):
+    """||Q^T Q - I||_F of the oracle's plain fp32 Householder QR (accumulation in
+    float, acc="f"): what an fp32 Householder QR of this matrix reaches."""
+    _, Qf = oracle.qr(A64, want_q=True, acc="f")
+    n = A64.shape[1]
+    return np.linalg.norm(Qf.T @ Qf - np.eye(n))
+
+
+def orth_bound(A64, bd, dt):
+    """north_star's 1e-5 (fp32) / 1e-13 (fp64) orthogonality bound.  SURVEY 9.1:
+    for fp32 and n > 192 an fp32 Householder QR itself exceeds 1e-5 (LAPACK
+    sgeqrf+sorgqr: 1.5e-5 at n = 512 ... 8.4e-5 at 8192), so there the bound is
+    3x the oracle's own fp32 value on the same matrix."""
+    n = A64.shape[1]
+    if dt == np.float32 and n > 192:
+        return max(bd["orth"], 3.0 * oracle_f_orth(A64))
+    return bd["orth"]
+
+
 def check_against_oracle(c, A, opts=None, C_cols=3):
     dt = A.dtype.type
     bd = BOUNDS[dt]
@@ -60,7 +79,7 @@ def check_against_oracle(c, A, opts=None, C_cols=3):
     nr = max(np.linalg.norm(Ron), 1e-300)
     assert np.linalg.norm(Rn - Ron) / nr <= bd["r"], "R vs oracle"
     assert np.linalg.norm(A64 - Q @ R) / max(np.linalg.norm(A64), 1e-300) <= bd["res"], "residual"
-    assert np.linalg.norm(Q.T @ Q - np.eye(n)) <= bd["orth"] * max(1, n / 192), "orthogonality"
+    assert np.linalg.norm(Q.T @ Q - np.eye(n)) <= orth_bound(A64, bd, dt), "orthogonality"
     # Q^T C: top n rows equal Q_thin^T C (sign-normalised); column norms preserved
     if C_cols:
         rng = np.random.default_rng(m + n)
@@ -108,10 +127,13 @@ def test_leaf_size_sweep(caqr, leaf_rows):
 
 
 @pytest.mark.parametrize("shape,nb", [((512, 512), 64), ((1000, 300), 0), ((2000, 130), 32),
-                                       ((700, 200), 96)])
+                                       ((700, 200), 96), ((3000, 256), 0), ((1024, 1024), 64)])
 @pytest.mark.parametrize("dtype", [np.float32, np.float64], ids=["f32", "f64"])
 def test_caqr_panel_loop(caqr, shape, nb, dtype):
-    """CAQR: TSQR panel groups + trailing update (Fig. 4), square-ish shapes."""
+    """CAQR: TSQR panel groups + trailing update (Fig. 4), square-ish
+    shapes, at north_star's unrelaxed R and residual bounds (fp32 LAPACK reaches
+    4.6-5.9e-7 on R and <= 7.1e-7 residual for square n <= 8192, SURVEY 8(c));
+    orthogonality per orth_bound."""
     A = workloads.gaussian(*shape, seed=11, dtype=dtype)
     opts = caqr.make_opts(panel_cols=nb) if nb else None
     m, n = shape
@@ -121,13 +143,77 @@ def test_caqr_panel_loop(caqr, shape, nb, dtype):
     Ro = oracle.qr(A64, want_q=False, acc=bd["acc"])
     Rn = oracle.normalize_signs(R)
     Ron = oracle.normalize_signs(Ro)
-    # square inputs are less well conditioned: scale the R bound by kappa-ish factor
-    kappa = np.linalg.cond(A64)
-    assert np.linalg.norm(Rn - Ron) / np.linalg.norm(Ron) <= max(bd["r"], 10 * kappa * np.finfo(dtype).eps)
-    assert np.linalg.norm(A64 - Q @ R) / np.linalg.norm(A64) <= bd["res"] * 4
-    # fp32 orthogonality grows ~ n^0.6; LAPACK itself exceeds 1e-5 for n >= 512
-    orth_tol = bd["orth"] if n <= 192 else 3 * np.finfo(dtype).eps * n * 10
-    assert np.linalg.norm(Q.T @ Q - np.eye(n)) <= max(orth_tol, bd["orth"])
+    assert np.linalg.norm(Rn - Ron) / np.linalg.norm(Ron) <= bd["r"]
+    assert np.linalg.norm(A64 - Q @ R) / np.linalg.norm(A64) <= bd["res"]
+    assert np.linalg.norm(Q.T @ Q - np.eye(n)) <= orth_bound(A64, bd, dtype)
+
+
+def test_caqr_2048_square_vs_oracle(caqr):
+    """Square CAQR (the C5 path: 64-wide panel groups, trailing update on the
+    tensor cores) at 2048 x 2048 against the oracle, unrelaxed R bound 1e-4."""
+    A = workloads.gaussian(2048, 2048, seed=3)
+    R, Q, Ad, ws = gpu_qr(caqr, A, caqr.make_opts(panel_cols=64))
+    A64 = A.astype(np.float64)
+    Ron = oracle.normalize_signs(oracle.qr(A64, want_q=False))
+    assert np.linalg.norm(oracle.normalize_signs(R) - Ron) / np.linalg.norm(Ron) <= 1e-4
+    assert np.linalg.norm(A64 - Q @ R) / np.linalg.norm(A64) <= 1e-5
+    assert np.linalg.norm(Q.T @ Q - np.eye(2048)) <= 3.0 * oracle_f_orth(A64)
+
+
+def test_c5_square_8192_properties(caqr):
+    """Config C5 (8192 x 8192 fp32, panel width 64) in its default plan: checks
+    that hold at any size, in fp64 on the device -- R^T R = A^T A and A = QR at
+    north_star's 1e-5, and ||Q^T Q - I||_F <= 3x the oracle's own fp32
+    Householder QR on an 8192^2 Gaussian (tests/golden/oracle_f_orth.json,
+    tools/make_golden_orth.py; the 1e-5 of north_star is infeasible
+    for any fp32 Householder QR at this n -- fp32 LAPACK: 8.4e-5)."""
+    import json
+    import os
+    with open(os.path.join(os.path.dirname(__file__), "golden", "oracle_f_orth.json")) as f:
+        orth_f = float(json.load(f)["8192"])
+    n = 8192
+    A = workloads.device_gaussian(n, n, seed=7, dtype=torch.float32, device="cuda").t()
+    A0 = A.clone()
+    R, ws = caqr.caqr_factor(A)
+    Q = caqr.caqr_form_q(A, ws)
+    torch.cuda.synchronize()
+    A64 = A0.double()
+    del A0
+    R64 = R.double()
+    G = A64.t() @ A64
+    assert (torch.linalg.norm(R64.t() @ R64 - G) / torch.linalg.norm(G)).item() <= 1e-5
+    del G
+    Q64 = Q.double()
+    del Q
+    assert (torch.linalg.norm(A64 - Q64 @ R64) / torch.linalg.norm(A64)).item() <= 1e-5
+    I = torch.eye(n, dtype=torch.float64, device="cuda")
+    assert torch.linalg.norm(Q64.t() @ Q64 - I).item() <= 3.0 * orth_f
+
+
+@pytest.mark.parametrize("name,dtype,tol", [("r_1000000x192_f32_seed0", np.float32, 1e-4),
+                                            ("r_200000x192_f64_seed1", np.float64, 1e-12)],
+                         ids=["C4-f32-1Mx192", "C4-f64-200kx192"])
+def test_full_size_r_vs_oracle_golden(caqr, name, dtype, tol):
+    """Config C4 at full size: the whole R (every element) against the oracle's R,
+    computed on the CPU by tools/make_golden.py (oracle only) from the same seeded
+    host input, in the bench's launch configuration (default plan).  fp32: oracle
+    in double; fp64: oracle in long double."""
+    import os
+    g = np.load(os.path.join(os.path.dirname(__file__), "golden", name + ".npz"))
+    m, n, seed = int(g["m"]), int(g["n"]), int(g["seed"])
+    A = workloads.gaussian(m, n, seed=seed, dtype=dtype)
+    R, _, Ad, ws = gpu_qr(caqr, A, want_q=False)
+    Ro = g["R"]
+    assert np.all(np.tril(R, -1) == 0)
+    err = np.linalg.norm(oracle.normalize_signs(R) - Ro) / np.linalg.norm(Ro)
+    assert err <= tol, err
+    # Q^T A = [R; 0]: top rows equal R, bottom rows vanish (relative to ||A||)
+    Cd = to_dev(caqr, A[:, :4])
+    caqr.caqr_apply_qt(Ad, ws, Cd)
+    QtA = Cd.cpu().numpy().astype(np.float64)
+    res = 1e-5 if dtype == np.float32 else 1e-13
+    assert np.linalg.norm(QtA[:n] - R[:, :4]) / np.linalg.norm(R[:, :4]) <= 10 * res
+    assert np.linalg.norm(QtA[n:]) / np.linalg.norm(A[:, :4].astype(np.float64)) <= 10 * res
 
 
 def test_deterministic(caqr):
@@ -619,3 +705,110 @@ def test_factor_host_errors(caqr):
         caqr.caqr_factor_host(torch.zeros(64, 100).t(), 4)  # 100 x 64 in 4 chunks: m/S < n
     with pytest.raises(ValueError):
         caqr.caqr_factor_host(torch.zeros(100, 4, device="cuda").t().contiguous().t(), 2)
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64], ids=["f32", "f64"])
+@pytest.mark.parametrize("P,m,n", [(2, 4000, 64), (3, 10001, 96), (8, 40000, 192), (8, 1600, 192)])
+def test_dist_combine_blocks_P_ranks(caqr, P, m, n, dtype):
+    """The post-all-gather half of caqr_dist_factor (caqr_dist_combine_blocks,
+    the code caqr_dist_factor runs after ncclAllGather) at P > 1, emulating P
+    ranks on one GPU: each row shard factored on its own, the local R's laid out
+    exactly as the all-gather leaves them (P contiguous n x n column-major
+    blocks in rank order, some with ldr != n copies), restacked + combined.  The
+    result must be the oracle's R of the whole matrix (uniqueness of R, S17),
+    and Q^T A through the local Q's and the combine's Q_c must be [R; 0]."""
+    from paper_conf_ipps_andersonbdk11_b200 import dist as cdist
+
+    tdt = torch.float32 if dtype == np.float32 else torch.float64
+    bd = BOUNDS[dtype]
+    A = workloads.gaussian(m, n, seed=100 + P, dtype=dtype)
+    blocks = torch.empty(P * n * n, dtype=tdt, device="cuda")
+    shards = []
+    for p in range(P):
+        s0, rows = cdist.shard_rows(m, P, p)
+        Ap = caqr.colmajor_empty(rows, n, tdt)
+        Ap.copy_(torch.from_numpy(A[s0:s0 + rows]))
+        Rp, wsp = caqr.caqr_factor(Ap)
+        # the send slot of rank p: its R as a contiguous column-major n x n block
+        blocks[p * n * n:(p + 1) * n * n].copy_(Rp.t().contiguous().reshape(-1))
+        shards.append((s0, rows, Ap, wsp))
+    R, gather, cws = caqr.caqr_dist_combine_blocks(blocks, P, n)
+    torch.cuda.synchronize()
+    Rn = R.cpu().double().numpy()
+    assert np.all(np.tril(Rn, -1) == 0)
+    A64 = A.astype(np.float64)
+    Ro = oracle.normalize_signs(oracle.qr(A64, want_q=False, acc=bd["acc"]))
+    assert np.linalg.norm(oracle.normalize_signs(Rn) - Ro) / np.linalg.norm(Ro) <= bd["r"]
+    # Q^T A: local Q_p^T A_p, top n rows of every shard stacked, then Q_c^T
+    k = 3
+    top = caqr.colmajor_empty(P * n, k, tdt)
+    bottom_sq = 0.0
+    for p, (s0, rows, Ap, wsp) in enumerate(shards):
+        Cp = to_dev(caqr, A[s0:s0 + rows, :k])
+        caqr.caqr_apply_qt(Ap, wsp, Cp)
+        top[p * n:(p + 1) * n].copy_(Cp[:n])
+        bottom_sq += float((Cp[n:].double() ** 2).sum())
+    caqr.caqr_combine_apply(gather, P, cws, top, trans=True)
+    T = top.cpu().double().numpy()
+    scale = np.linalg.norm(A64[:, :k])
+    assert np.linalg.norm(T[:n] - Rn[:, :k]) / scale <= 10 * bd["res"]
+    assert np.sqrt(bottom_sq + np.linalg.norm(T[n:]) ** 2) / scale <= 10 * bd["res"]
+
+
+def test_dist_combine_blocks_errors(caqr):
+    blocks = torch.zeros(2 * 4 * 4, device="cuda")
+    with pytest.raises(caqr.CaqrError):
+        caqr.caqr_dist_combine_blocks(blocks, 0, 4)          # P < 1
+    with pytest.raises(caqr.CaqrError):
+        caqr.caqr_dist_combine_blocks(blocks, 2, 4, cws=torch.empty(8, dtype=torch.uint8, device="cuda"))
+
+
+@pytest.mark.parametrize("dual", ["0", "1"])
+@pytest.mark.parametrize("m,n,S,nb", [(30000, 192, 6, 0), (20000, 130, 4, 64), (9000, 96, 3, 32)])
+def test_factor_host_dual_and_panel_groups(caqr, m, n, S, nb, dual, monkeypatch):
+    """caqr_factor_host with both stream policies (CAQR_HOST_DUAL: odd chunks on
+    the library's second stream or all on the caller's) and with chunks that run
+    the CAQR panel loop (panel_cols < n: the shared early-start side stream):
+    R against the oracle and bitwise identical between the two policies."""
+    monkeypatch.setenv("CAQR_HOST_DUAL", dual)
+    A = workloads.gaussian(m, n, seed=m + S, dtype=np.float32)
+    Ah = torch.empty((n, m), dtype=torch.float32, pin_memory=True).t()
+    Ah.copy_(torch.from_numpy(A))
+    opts = caqr.make_opts(panel_cols=nb) if nb else None
+    Ad, R, ws = caqr.caqr_factor_host(Ah, S, opts=opts)
+    torch.cuda.synchronize()
+    R = R.cpu().numpy().astype(np.float64)
+    Ro = oracle.normalize_signs(oracle.qr(A.astype(np.float64), want_q=False))
+    assert np.linalg.norm(oracle.normalize_signs(R) - Ro) / np.linalg.norm(Ro) <= 1e-4
+    monkeypatch.setenv("CAQR_HOST_DUAL", "1" if dual == "0" else "0")
+    _, R2, _ = caqr.caqr_factor_host(Ah, S, opts=opts)
+    torch.cuda.synchronize()
+    assert np.array_equal(R, R2.cpu().numpy().astype(np.float64))
+
+
+def test_concurrent_caqr_calls_two_threads(caqr):
+    """Two host threads factoring different matrices through the CAQR panel loop
+    (n > 256: early-start overlap on the per-device side stream) at once, each
+    on its own stream: both R's match their single-threaded results bitwise."""
+    import threading
+
+    mats = [workloads.gaussian(3000, 300, seed=s) for s in (1, 2)]
+    ref = [gpu_qr(caqr, M, want_q=False)[0] for M in mats]
+    out = [None, None]
+
+    def work(i):
+        st = torch.cuda.Stream()
+        with torch.cuda.stream(st):
+            for _ in range(5):
+                Ad = to_dev(caqr, mats[i])
+                R, _ = caqr.caqr_factor(Ad, stream=st)
+            st.synchronize()
+            out[i] = R.cpu().numpy().astype(np.float64)
+
+    th = [threading.Thread(target=work, args=(i,)) for i in range(2)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    for i in range(2):
+        assert np.array_equal(out[i], ref[i])
