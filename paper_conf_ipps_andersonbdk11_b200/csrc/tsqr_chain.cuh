@@ -929,11 +929,14 @@ tsqr_chain_kernel(Geom g, float* __restrict__ A, float* __restrict__ Tws, int* _
                         // ---- epilogue: C -= dC (rows: TMEM lanes), store tile rows + slot rows ----
                         {
                             auto rows_out = [&](int row, const float (&v)[16]) {
+                                const bool rok = row < h && !(leaf && row < hr0);
+                                float* gp = A + cb0 * lda + s + row;  // column cb0, this row; += lda per column
 #pragma unroll
                                 for (int n = 0; n < CW; ++n) {
                                     const float cn = fmaf(-v[n], wscale[n], Cs[(size_t)n * VP + row]);
                                     Cs[(size_t)n * VP + row] = cn;
-                                    if (n < ncb && row < h && !(leaf && row < hr0)) A[(cb0 + n) * lda + s + row] = cn;
+                                    if (rok && n < ncb) __stcg(gp, cn);
+                                    gp += lda;
                                 }
                             };
                             float v[16];

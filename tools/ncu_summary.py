@@ -26,6 +26,11 @@ raw = list(csv.reader(io.StringIO(run("--page", "raw", "--csv"))))
 if len(raw) > 2:
     rh, units, vals = raw[0], raw[1], raw[2]
     for k in ["dram__bytes_read.sum", "dram__bytes_write.sum", "sm__inst_executed_pipe_fma.avg.pct_of_peak_sustained_active",
+              "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active",
+              "sm__pipe_tensor_op_hmma_cycles_active.avg.pct_of_peak_sustained_active",
+              "sm__inst_executed_pipe_uma.avg.pct_of_peak_sustained_active",
+              "sm__warps_active.avg.pct_of_peak_sustained_active",
+              "smsp__average_warps_issue_stalled_barrier_per_issue_active.ratio",
               "sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active",
               "smsp__average_warp_latency_issue_stalled_barrier", "sm__throughput.avg.pct_of_peak_sustained_elapsed",
               "lts__t_bytes.sum", "l1tex__data_bank_conflicts_pipe_lsu_mem_shared.sum"]:
