@@ -27,8 +27,11 @@
  *     DEVICE pointers (cudaMalloc'd or torch CUDA storage) on the current device,
  *     except A_host of caqr_factor_host_* (host memory, by name).
  *   - Calls only enqueue work on `stream` (0 = legacy default stream); they never
- *     synchronise the device, never allocate device memory, and are safe to
- *     capture into a CUDA graph.  They are reentrant; the only process state is
+ *     synchronise the device, never allocate device memory, and can be captured
+ *     into a CUDA graph (tests/test_gpu_parity.py test_cuda_graph_capture:
+ *     factor, apply_qt, form_q, the CAQR loop with its early-start fork/join).
+ *     They are reentrant (calls from several host threads: test_concurrent_
+ *     caqr_calls_two_threads); the only process state is
  *     a lazily-filled per-device attribute cache and the lazily-created side
  *     stream (CAQR early start) and copy + second compute stream
  *     (caqr_factor_host_*) per device.

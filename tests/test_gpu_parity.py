@@ -812,3 +812,42 @@ def test_concurrent_caqr_calls_two_threads(caqr):
         t.join()
     for i in range(2):
         assert np.array_equal(out[i], ref[i])
+
+
+@pytest.mark.parametrize("m,n", [(100_000, 192), (3000, 300)])
+def test_cuda_graph_capture(caqr, m, n):
+    """The header's claim that every call only enqueues work on its stream:
+    factor + apply_qt + form_q captured into one CUDA graph (for n = 300 the
+    CAQR loop with its early-start fork to the library's side stream and the
+    join back), replayed twice on a freshly restored A: R, Q^T C and Q bitwise
+    equal to the eager calls."""
+    A = workloads.gaussian(m, n, seed=9)
+    Ad = to_dev(caqr, A)
+    A0 = Ad.clone()
+    C0 = to_dev(caqr, A[:, :3])
+    R, ws = caqr.caqr_factor(Ad)
+    C = C0.clone()
+    caqr.caqr_apply_qt(Ad, ws, C)
+    Q = caqr.caqr_form_q(Ad, ws)
+    torch.cuda.synchronize()
+    R_e, C_e, Q_e = R.clone(), C.clone(), Q.clone()
+    st = torch.cuda.Stream()
+    st.wait_stream(torch.cuda.current_stream())
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.stream(st):
+        Ad.copy_(A0)
+        C.copy_(C0)
+        torch.cuda.synchronize()
+        with torch.cuda.graph(g, stream=st):
+            caqr.caqr_factor(Ad, R=R, ws=ws, stream=st)
+            caqr.caqr_apply_qt(Ad, ws, C, stream=st)
+            caqr.caqr_form_q(Ad, ws, Q=Q, stream=st)
+    for _ in range(2):
+        Ad.copy_(A0)
+        C.copy_(C0)
+        R.zero_()
+        Q.zero_()
+        torch.cuda.synchronize()
+        g.replay()
+        torch.cuda.synchronize()
+        assert torch.equal(R, R_e) and torch.equal(C, C_e) and torch.equal(Q, Q_e)
