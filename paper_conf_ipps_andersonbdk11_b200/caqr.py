@@ -502,19 +502,6 @@ def geqrf_flops(m: int, n: int) -> float:
     return 2.0 * m * n * n - 2.0 * n ** 3 / 3.0
 
 
-def qr_host(A_host, opts=None, stream=None, pinned_out=None):
-    """End-to-end public call from host memory: H2D copy of A (pinned host
-    tensor, column-major), caqr_factor on the GPU, D2H copy of R.  Returns the
-    host R (and leaves the device factorisation in the returned tuple)."""
-    torch = _torch()
-    A_dev = colmajor_empty(A_host.shape[0], A_host.shape[1], A_host.dtype, "cuda")
-    A_dev.copy_(A_host, non_blocking=True)
-    R, ws = caqr_factor(A_dev, opts=opts, stream=stream)
-    out = pinned_out if pinned_out is not None else torch.empty(R.shape, dtype=R.dtype, pin_memory=True)
-    out.copy_(R, non_blocking=True)
-    return out, A_dev, ws
-
-
 # ---- launch tracing (profiling aid) -----------------------------------------
 def caqr_trace_begin(capacity: int = 1 << 16) -> None:
     _check("caqr_trace_begin", lib().caqr_trace_begin(capacity))

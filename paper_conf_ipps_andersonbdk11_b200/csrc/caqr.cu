@@ -492,15 +492,6 @@ static unsigned long long* prof_buffer() {
     return g_prof;
 }
 
-// CAQR_LA=1 selects the look-ahead (two-role, 1 CTA/SM) fp32 fused kernel.
-// Off by default: measured on B200 at 1M x 192 it loses to two independent
-// single-role CTAs per SM (9.5 ms with a matched 148-chain plan vs 7.9 ms).
-static inline int la_policy() {
-    const char* e = getenv("CAQR_LA");
-    return (e && e[0] == '1') ? 1 : 0;
-}
-
-// The whole TSQR of a group (leaves + every tree level) in one persistent launch.
 template <typename T>
 static int launch_fused(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, cudaStream_t s) {
     const int nl = tree_levels(G.P);
@@ -516,20 +507,6 @@ static int launch_fused(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, 
         by = 2.0 * mr * nc * sizeof(T);
     }
     bool done = false;
-    if constexpr (sizeof(T) == 4) {
-        if (la_policy()) {
-            done = true;
-            const size_t smem = la_smem_bytes<T>();
-            if (e == cudaSuccess) e = allow_smem(tsqr_la_kernel<T>, smem);
-            if (e == cudaSuccess) {
-                const int64_t grid = std::min<int64_t>(total, num_sms());
-                TraceScope ts(K_TSQR_FUSED, fl, by, s);
-                tsqr_la_kernel<T><<<(unsigned)grid, 2 * kThreads, smem, s>>>(G, A, Tws, sync, nl,
-                                                                           do_leaves ? 1 : 0);
-                e = cudaGetLastError();
-            }
-        }
-    }
     if (!done) {
         const size_t smem = fused_smem_bytes<T>();
         if (e == cudaSuccess) e = allow_smem(tsqr_fused_kernel<T>, smem);

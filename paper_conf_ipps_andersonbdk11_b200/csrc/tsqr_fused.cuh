@@ -1298,194 +1298,3 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
 }
 
 }  // namespace caqr
-
-// ===========================================================================
-// Look-ahead variant (fp32): one CTA of 512 threads per SM, two roles.
-//   F (warps 0-7, named barrier 1): stage + factor the NEXT panel (WB4), its
-//     T, and write it out;
-//   U (warps 8-15, named barrier 2): apply the CURRENT panel's block
-//     reflector to the node's trailing column blocks.
-// Per panel p: U first updates block p+1 (the next panel's columns; F waits),
-// then F factors panel p+1 while U updates blocks >= p+2 -- the classic
-// look-ahead, so the latency-bound panel factorization overlaps the GEMM-like
-// trailing update instead of alternating with it.
-// ===========================================================================
-namespace caqr {
-
-template <typename T>
-struct LaSmem {
-    T *PA, *PB, *Cs, *Wp, *WpF, *TA, *TB, *WU, *WF, *tauA, *tauB, *TbF, *scrF;
-};
-
-template <typename T>
-__host__ __device__ inline size_t la_smem_elems(int RGP) {
-    return 3 * 32 * (size_t)RGP + 2 * 4 * 32 * kTS + 4 * 32 * kTS + 64 + 128 + kWarps * (32 * 20 + 16);
-}
-template <typename T>
-inline size_t la_smem_bytes() {
-    return sizeof(T) * la_smem_elems<T>(fused_col_stride<T>(kFusedMaxRows)) + 64;
-}
-
-template <typename T>
-__device__ __forceinline__ void la_factor_panel(const Grp& GF, const Geom& g, T* A, T* Tws, int level,
-                                                int64_t node, int kt, int p, T* P, T* Tt, T* tau, T* WpF,
-                                                T* WF, T* Tb, T* scr, int RGP) {
-    const int wp = min(kPW, g.ncols - 32 * p);
-    const NodeRows nr = node_rows(g, level, node, p, wp, kt);
-    const int RG = nr.n0 + nr.n1;
-    const int R32 = (RG + 31) & ~31;
-    const int64_t c0 = g.col0 + 32 * p;
-    stage_cols(GF, P, RGP, R32, static_cast<const T*>(A), g.lda, c0, wp, nr, RG, true, p);
-    if (GF.tid < 32) tau[GF.tid] = T(0);
-    gsync(GF);
-    factor_panel_wb4<T>(GF, P, RGP, RG, wp, tau, Tb, scr);
-    {
-        const int warp = GF.tid >> 5, lane = GF.tid & 31;
-        for (int jj = warp; jj < 32; jj += kWarps) {
-            T* col = A + (c0 + jj) * g.lda;
-            T* pc = P + (size_t)jj * RGP;
-            for (int r = lane; r < R32; r += 32) {
-                const bool in = r < RG && jj < wp;
-                const T val = pc[padr<T>(r)];
-                if (in && panel_entry_stored(nr, r, jj, p)) col[gathered_row(nr, r)] = val;
-                pc[padr<T>(r)] = in ? v_entry<T>(nr, r, jj, p, val) : T(0);
-            }
-        }
-    }
-    gsync(GF);
-    gemm_vtc(GF, P, P, RGP, R32, WpF, WF);  // G = V^T V
-    build_t(GF, WF, tau, wp, Tt);
-    gsync(GF);
-    T* tb = Tws + nr.tblk * (kPW * kPW);
-    for (int e = GF.tid; e < kPW * kPW; e += kThreads) tb[e] = Tt[(e & 31) * kTS + (e >> 5)];
-}
-
-template <typename T>
-__device__ __forceinline__ void la_update_block(const Grp& GU, const Geom& g, T* A, const NodeRows& nr, int p,
-                                                int wp, int64_t cb0, int ncb, const T* P, const T* Tt, T* Cs,
-                                                T* Wp, T* WU, int RGP) {
-    const int RG = nr.n0 + nr.n1;
-    const int R32 = (RG + 31) & ~31;
-    stage_cols(GU, Cs, RGP, R32, static_cast<const T*>(A), g.lda, cb0, ncb, nr, RG, false, p);
-    gsync(GU);
-    if constexpr (sizeof(T) == 4)
-        gemm_vtc_mma<true>(GU, P, Cs, RGP, R32, Wp, WU);
-    else
-        gemm_vtc(GU, P, Cs, RGP, R32, Wp, WU);
-    apply_block(GU, P, Cs, Tt, WU, RGP, R32, RG, wp, 1, nr, A, g.lda, cb0, ncb);
-}
-
-template <typename T>
-__global__ void __launch_bounds__(2 * kThreads, 1)
-tsqr_la_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int nlevels, int do_leaves) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    const int RGP = fused_col_stride<T>(kFusedMaxRows);
-    T* base = reinterpret_cast<T*>(smem_raw);
-    T* PA = base;
-    T* PB = PA + 32 * (size_t)RGP;
-    T* Cs = PB + 32 * (size_t)RGP;
-    T* Wp = Cs + 32 * (size_t)RGP;
-    T* WpF = Wp + 4 * 32 * kTS;
-    T* TA = WpF + 4 * 32 * kTS;
-    T* TB = TA + 32 * kTS;
-    T* WU = TB + 32 * kTS;
-    T* WF = WU + 32 * kTS;
-    T* tauA = WF + 32 * kTS;
-    T* tauB = tauA + 32;
-    T* TbF = tauB + 32;
-    T* scrF = TbF + 128;
-    __shared__ int s_task;
-    const bool isF = threadIdx.x < kThreads;
-    const Grp GF{(int)threadIdx.x, 1}, GU{(int)threadIdx.x - kThreads, 2};
-    int* ticket = sync;
-    int* flags = sync + 32;
-    const int64_t leaf_tasks = do_leaves ? g.P : 0;
-    int64_t total = leaf_tasks;
-    for (int l = 0; l < nlevels; ++l) {
-        const int64_t h = int64_t(1) << l;
-        total += (g.P - 1 >= h) ? (g.P - 1 - h) / (2 * h) + 1 : 0;
-    }
-    for (;;) {
-        __syncthreads();
-        if (threadIdx.x == 0) s_task = atomicAdd(ticket, 1);
-        __syncthreads();
-        const int64_t task = s_task;
-        if (task >= total) break;
-        int level = -1;
-        int64_t node = task;
-        if (task >= leaf_tasks) {
-            node = task - leaf_tasks;
-            level = 0;
-            for (;;) {
-                const int64_t h = int64_t(1) << level;
-                const int64_t nm = (g.P - 1 >= h) ? (g.P - 1 - h) / (2 * h) + 1 : 0;
-                if (node < nm) break;
-                node -= nm;
-                ++level;
-            }
-        }
-        int64_t slot_a, slot_b = -1;
-        int ver_a = 0, ver_b = 0;
-        if (level < 0) {
-            slot_a = node;
-        } else {
-            slot_a = node << (level + 1);
-            slot_b = slot_a + (int64_t(1) << level);
-            ver_a = expected_version(slot_a, level, g.P, do_leaves);
-            ver_b = expected_version(slot_b, level, g.P, do_leaves);
-        }
-        const int my_ver = level < 0 ? 1 : level + 2;
-        const int64_t ntile = level < 0 ? min(g.K, g.L - node * g.K) : 1;
-        auto wait_children = [&](int p) {  // F thread 0; then F barrier
-            if (level >= 0 && GF.tid == 0) {
-                const int* fa = flags + slot_a * g.npan + p;
-                const int* fb = flags + slot_b * g.npan + p;
-                while (ld_acquire(fa) < ver_a) __nanosleep(64);
-                while (ld_acquire(fb) < ver_b) __nanosleep(64);
-            }
-            gsync(GF);
-        };
-        for (int kt = 0; kt < ntile; ++kt) {
-            T *Pc = PA, *Pn = PB, *Tc = TA, *Tn = TB, *tc = tauA, *tn = tauB;
-            if (isF) {
-                wait_children(0);
-                la_factor_panel(GF, g, A, Tws, level, node, kt, 0, Pc, Tc, tc, WpF, WF, TbF, scrF, RGP);
-            }
-            __syncthreads();
-            for (int p = 0; p < g.npan; ++p) {
-                const int wp = min(kPW, g.ncols - 32 * p);
-                const bool has_next = p + 1 < g.npan;
-                const NodeRows nr = node_rows(g, level, node, p, wp, kt);
-                const int64_t c0 = g.col0 + 32 * p, tend = g.col0 + g.ncols;
-                // step 1: U brings the next panel's columns up to date
-                if (!isF && has_next) {
-                    const int64_t cb0 = c0 + 32;
-                    la_update_block(GU, g, A, nr, p, wp, cb0, (int)(tend - cb0 < 32 ? tend - cb0 : 32), Pc, Tc, Cs,
-                                    Wp, WU, RGP);
-                }
-                __syncthreads();
-                // step 2: F factors panel p+1 while U updates the far blocks
-                if (isF) {
-                    if (has_next) {
-                        wait_children(p + 1);
-                        la_factor_panel(GF, g, A, Tws, level, node, kt, p + 1, Pn, Tn, tn, WpF, WF, TbF, scrF,
-                                        RGP);
-                    }
-                } else {
-                    for (int64_t cb0 = c0 + 64; cb0 < tend; cb0 += 32)
-                        la_update_block(GU, g, A, nr, p, wp, cb0, (int)(tend - cb0 < 32 ? tend - cb0 : 32), Pc, Tc,
-                                        Cs, Wp, WU, RGP);
-                }
-                __threadfence();
-                __syncthreads();
-                if (threadIdx.x == 0 && kt == ntile - 1) st_release(flags + slot_a * g.npan + p, my_ver);
-                T* t;
-                t = Pc; Pc = Pn; Pn = t;
-                t = Tc; Tc = Tn; Tn = t;
-                t = tc; tc = tn; tn = t;
-            }
-        }
-    }
-}
-
-}  // namespace caqr

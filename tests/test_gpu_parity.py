@@ -400,13 +400,6 @@ def test_fused_and_split_agree(caqr, monkeypatch):
     assert np.linalg.norm(R1 - R2) / np.linalg.norm(R1) <= 1e-5
 
 
-def test_lookahead_kernel(caqr, monkeypatch):
-    """The look-ahead (two-role) fp32 fused kernel: same plan, same R to rounding."""
-    monkeypatch.setenv("CAQR_LA", "1")
-    A = workloads.gaussian(70000, 192, seed=12)
-    check_against_oracle(caqr, A, opts=caqr.make_opts(leaf_rows=224), C_cols=2)
-
-
 @pytest.mark.parametrize("m,n", [(600_000, 16), (2_100_000, 8), (530_000, 3)])
 def test_skinny_chains(caqr, m, n):
     """Skinny fp32 panels (n <= 16) go to the streaming warp-per-chain kernel;
