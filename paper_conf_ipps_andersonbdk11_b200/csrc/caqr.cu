@@ -172,11 +172,13 @@ static inline int64_t merges_at(int64_t L, int level) {
     const int64_t h = int64_t(1) << level;
     return (L - 1 >= h) ? (L - 1 - h) / (2 * h) + 1 : 0;
 }
-// Workspace of one panel group: T blocks [2][L][npan][32][32] (leaf T's, then
-// merge T's indexed by the merge's right member), then the fused kernel's
+// Workspace of one panel group: T blocks [L + P][npan][32][32] (tile T's, then
+// merge T's indexed by the merge's right member's slot), then the fused kernel's
 // ticket + per-(slot, panel) ready flags.
 static inline size_t group_t_bytes(const Geom& G, size_t es) {
-    return (size_t)2 * G.L * G.npan * kPW * kPW * es;
+    // one 32 x 32 T per (tile, panel), then one per (merge, panel) indexed by
+    // the merge's right member (a chain slot, < P)
+    return (size_t)(G.L + G.P) * G.npan * kPW * kPW * es;
 }
 static inline size_t group_sync_bytes(const Geom& G) {
     int64_t ints = 32 + G.L * G.npan;

@@ -97,7 +97,7 @@ __device__ __forceinline__ NodeRows node_rows(const Geom& g, int level, int64_t 
         nr.n1 = (int32_t)(32 * p + wp < hb ? 32 * p + wp : hb);
         nr.seg0_tri = 1;
         nr.seg1_upper = 1;
-        nr.tblk = (g.L + bb * g.K) * g.npan + p;
+        nr.tblk = (g.L + bb) * g.npan + p;  // merges: indexed by the right member's slot
     }
     return nr;
 }

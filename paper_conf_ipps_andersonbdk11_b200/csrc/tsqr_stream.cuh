@@ -374,7 +374,7 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
             for (int i = 0; i < NC; ++i)
                 if (i <= k && i < hb) bb[i] = rb[i];
         }
-        stream_write_t<T, NC>(on, k, G, LDR, tau, wp, Tws + ((g.L + sb * g.K) * g.npan) * (kPW * kPW));
+        stream_write_t<T, NC>(on, k, G, LDR, tau, wp, Tws + ((g.L + sb) * g.npan) * (kPW * kPW));
     };
 
     // ---- the chain: tiles chain*K .., leaf first; R stays in W.R ----------
@@ -556,7 +556,7 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
                         if (i <= k && i < hb) bb[i] = rc.V[k][i];
                 }
                 stream_write_t<T, NC>(k < NC, k, &rc.G[0][0], NC, rc.tau, wp,
-                                      Tws + ((g.L + sb * g.K) * g.npan) * (kPW * kPW));
+                                      Tws + ((g.L + sb) * g.npan) * (kPW * kPW));
             }
         }
     }

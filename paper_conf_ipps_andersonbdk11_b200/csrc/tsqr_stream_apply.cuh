@@ -162,7 +162,7 @@ stream_apply_tree_kernel(Geom g, const float* __restrict__ A, const float* __res
     const int64_t a = node << (level + 1), b = a + hl;
     const int64_t ra = g.row0 + a * g.bm, rb = g.row0 + b * g.bm;
     const int nbr = (int)min64(min64(g.b, g.mrows - b * g.bm), wp);  // rows of R_b's slot
-    const float* tb = Tws + ((g.L + b * g.K) * g.npan) * (kPW * kPW);
+    const float* tb = Tws + ((g.L + b) * g.npan) * (kPW * kPW);
     for (int e = lane; e < NC * NC; e += 32) {
         const int i = e % NC, j = e / NC;
         s_V[warp][i][j] = (i <= j && i < nbr && j < wp) ? __ldcg(A + (g.col0 + j) * g.lda + rb + i) : 0.f;

@@ -35,10 +35,12 @@ def test_sass_is_sm100a():
 
 
 def test_workspace_bytes(L):
-    # one T block (32x32) per (leaf, panel) and per (merge, panel): 2*L*npan*1024 elems,
-    # plus the fused kernel's ticket + (slot, panel) flags: (32 + L*npan) ints, 256-B rounded
-    def ws(L, npan, es):
-        return 2 * L * npan * 1024 * es + -(-(32 + L * npan) * 4 // 256) * 256
+    # one T block (32x32) per (tile, panel) and per (merge, panel), the merges indexed
+    # by their right member's slot (< P chains): (L + P)*npan*1024 elems, plus the
+    # fused kernel's ticket + (slot, panel) flags: (32 + L*npan) ints, 256-B rounded
+    def ws(L, npan, es, P=None):
+        P = L if P is None else P
+        return (L + P) * npan * 1024 * es + -(-(32 + L * npan) * 4 // 256) * 256
     # default tile height 224 (n <= 224): 4096 rows -> 19 tiles, 1M rows -> 4465 tiles;
     # skinny fp32 (n <= 16, m >= 1024: the warp-per-chain streaming kernel) uses
     # 256 (n <= 8) / 128-row tiles and a cross-CTA exchange area in the flag
@@ -48,7 +50,7 @@ def test_workspace_bytes(L):
     sync = max(32 + 32, 64 + ((nct * 16 * 16 + 31) & ~31) + 16 * nct)
     assert caqr.caqr_workspace_bytes(4096, 16) == 2 * 32 * 1024 * 4 + -(-sync * 4 // 256) * 256
     assert caqr.caqr_workspace_bytes(4096, 16, caqr.CAQR_F64) == ws(19, 1, 8)
-    assert caqr.caqr_workspace_bytes(1_000_000, 192) == ws(4465, 6, 4)
+    assert caqr.caqr_workspace_bytes(1_000_000, 192) == ws(4465, 6, 4, P=280)  # chains of 16 tiles
     assert caqr.caqr_workspace_bytes(4096, 16, 0, caqr.make_opts(leaf_rows=256)) == ws(16, 1, 4)
     assert caqr.caqr_workspace_bytes(10, 11) == 0  # n > m
     assert caqr.caqr_workspace_bytes(-1, 1) == 0
