@@ -76,6 +76,12 @@ static inline bool stream16_policy() {
     const char* e = getenv("CAQR_STREAM16");
     return e && e[0] == '1';
 }
+// n <= 8 panels on 256-row tiles: 16 warps per SM with one tile buffer each
+// (default) or 8 warps with two (CAQR_STREAM_W16B=0).
+static inline bool stream_w16b_policy() {
+    const char* e = getenv("CAQR_STREAM_W16B");
+    return !(e && e[0] == '0');
+}
 
 struct Plan {
     int64_t m = 0, n = 0;
@@ -126,7 +132,8 @@ static int make_plan(int64_t m, int64_t n, int dtype, const caqr_opts* o, int op
     pl->skinny = dtype == CAQR_F32 && n <= 16 && nb >= n && m >= skinny_min_m;
     // streaming kernel: one chain per warp, 8 warps per SM (148 SMs)
     const bool s16 = pl->skinny && n <= 8 && stream16_policy();
-    pl->chain_target = pl->skinny ? (s16 ? 2 * kStreamChains : kStreamChains) : kChainTarget;
+    const bool w16 = pl->skinny && n <= 8 && (s16 || stream_w16b_policy());
+    pl->chain_target = pl->skinny ? (w16 ? 2 * kStreamChains : kStreamChains) : kChainTarget;
     if (const char* e = getenv("CAQR_CHAIN_TARGET"))  // diagnostics: chains per group (tile sweep)
         pl->chain_target = std::max<int64_t>(1, atoll(e));
     // fp32 whole-width groups (16 < n <= 256): the chain kernel (tsqr_chain.cuh),
@@ -624,10 +631,10 @@ static int launch_skinny(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves,
 
 // Streaming skinny TSQR (tsqr_stream.cuh): n <= 16, tiles of 256 (n <= 8) or
 // 128 rows, one chain per warp, 8 warps per CTA; true in *done if launched.
-template <typename T, int NC, int RPL, int NW = 8>
+template <typename T, int NC, int RPL, int NW = 8, int NBUF = 2>
 static cudaError_t launch_stream_nc(const Geom& G, T* A, T* Tws, int* sync, bool vec, cudaStream_t s) {
     const unsigned grid = (unsigned)ceil_div(G.P, NW);
-    const size_t smem = stream_smem_bytes<T, NC, RPL, NW>(grid);
+    const size_t smem = stream_smem_bytes<T, NC, RPL, NW, NBUF>(grid);
     const int nl = tree_levels(G.P);
     cudaError_t e;
     unsigned long long* prof = prof_buffer();
@@ -635,13 +642,13 @@ static cudaError_t launch_stream_nc(const Geom& G, T* A, T* Tws, int* sync, bool
     const int dbg = dbe ? atoi(dbe) : 0;
     if (prof) cudaMemsetAsync(prof, 0xff, sizeof(unsigned long long), s);  // [0] is a running min
     if (vec) {
-        e = allow_smem(tsqr_stream_kernel<T, NC, RPL, NW, true>, smem);
+        e = allow_smem(tsqr_stream_kernel<T, NC, RPL, NW, NBUF, true>, smem);
         if (e == cudaSuccess)
-            tsqr_stream_kernel<T, NC, RPL, NW, true><<<grid, 32 * NW, smem, s>>>(G, A, Tws, sync, nl, prof, dbg);
+            tsqr_stream_kernel<T, NC, RPL, NW, NBUF, true><<<grid, 32 * NW, smem, s>>>(G, A, Tws, sync, nl, prof, dbg);
     } else {
-        e = allow_smem(tsqr_stream_kernel<T, NC, RPL, NW, false>, smem);
+        e = allow_smem(tsqr_stream_kernel<T, NC, RPL, NW, NBUF, false>, smem);
         if (e == cudaSuccess)
-            tsqr_stream_kernel<T, NC, RPL, NW, false><<<grid, 32 * NW, smem, s>>>(G, A, Tws, sync, nl, prof, dbg);
+            tsqr_stream_kernel<T, NC, RPL, NW, NBUF, false><<<grid, 32 * NW, smem, s>>>(G, A, Tws, sync, nl, prof, dbg);
     }
     return e == cudaSuccess ? cudaGetLastError() : e;
 }
@@ -653,13 +660,17 @@ static int launch_stream(const Geom& G, T* A, T* Tws, int* sync, cudaStream_t s,
         const bool nc8 = G.ncols <= 8 && G.b == 256, nc16 = G.ncols <= 16 && G.b == 128;
         if (!nc8 && !nc16) return 0;
         const bool w16 = G.ncols <= 8 && G.b == 128;  // 16 warps x 128-row tiles (CAQR_STREAM16)
+        // 16 warps x 256-row tiles, one buffer each, once there are more
+        // tiles than 8 warps per SM would take (fewer: 8 warps, less tree)
+        const bool w16b = nc8 && G.L > kStreamChains && stream_w16b_policy();
         // the CTAs' R's travel through the workspace's flag area
-        const int64_t nct = ceil_div(G.P, w16 ? 16 : 8);
+        const int64_t nct = ceil_div(G.P, (w16 || w16b) ? 16 : 8);
         // (plus one arrival counter per (cross-CTA level, CTA))
         const int64_t rx = (nc8 || w16) ? stream_rx_ints<T, 8>(nct) : stream_rx_ints<T, 16>(nct);
         if ((64 + rx + (int64_t)tree_levels(G.P) * nct) * (int64_t)sizeof(int) > (int64_t)group_sync_bytes(G)) return 0;
-        if ((nc8 ? stream_smem_bytes<T, 8, 8, 8>(nct)
-                 : w16 ? stream_smem_bytes<T, 8, 4, 16>(nct) : stream_smem_bytes<T, 16, 4, 8>(nct)) > 220 * 1024)
+        if ((w16b  ? stream_smem_bytes<T, 8, 8, 16, 1>(nct)
+             : nc8 ? stream_smem_bytes<T, 8, 8, 8>(nct)
+             : w16 ? stream_smem_bytes<T, 8, 4, 16>(nct) : stream_smem_bytes<T, 16, 4, 8>(nct)) > 220 * 1024)
             return 0;
         // 16-byte cp.async needs every tile column start 16-byte aligned
         const bool vec = (reinterpret_cast<uintptr_t>(A) % 16 == 0) && (G.lda % 4 == 0) && (G.row0 % 4 == 0);
@@ -672,7 +683,8 @@ static int launch_stream(const Geom& G, T* A, T* Tws, int* sync, cudaStream_t s,
                 by = 2.0 * mr * nc * sizeof(T);
             }
             TraceScope ts(K_TSQR_SKINNY, fl, by, s);
-            e = nc8   ? launch_stream_nc<T, 8, 8>(G, A, Tws, sync, vec, s)
+            e = w16b  ? launch_stream_nc<T, 8, 8, 16, 1>(G, A, Tws, sync, vec, s)
+                : nc8 ? launch_stream_nc<T, 8, 8>(G, A, Tws, sync, vec, s)
                 : w16 ? launch_stream_nc<T, 8, 4, 16>(G, A, Tws, sync, vec, s)
                       : launch_stream_nc<T, 16, 4>(G, A, Tws, sync, vec, s);
         }

@@ -78,15 +78,17 @@ __device__ __forceinline__ void householder_scalars(T al, T sg, bool live, T& ta
 }
 
 // Per-warp shared state.
-template <typename T, int NC, int B>
+// NBUF = 2: double-buffered tile; NBUF = 1: one buffer, refilled as soon as
+// the warp has the current tile in registers (halves the shared memory, so
+// 16 warps of 256-row tiles fit per SM).
+template <typename T, int NC, int B, int NBUF = 2>
 struct alignas(16) StreamWarp {
-    T buf[2][NC][B];   // double-buffered tile (column-major, B rows)
+    T buf[NBUF][NC][B];  // tile buffer(s) (column-major, B rows)
     T R[NC][NC + 1];   // chain / subtree R, R[j][k] (upper)
     T G[NC][NC + 1];   // Gram entries G[a][j] = v_a^T v_j (a < j)
     T Rs[NC][NC + 1];  // a sibling CTA's R (cross-CTA merges)
     T tau[NC];
     T red[32];         // all-reduce scratch
-    T bc[2 * NC + 4];  // merge broadcast: v_j, tau, ...
 };
 
 // T (compact WY, xLARFT forward/columnwise) from tau and the Gram entries
@@ -154,8 +156,8 @@ __device__ __forceinline__ void stream_issue_tile(const Geom& g, const T* A, int
 // Leaf (kt == 0) or chain step (kt > 0) on the registers x[c][i] = row
 // lane + 32 i of column c.  Leaf: R ends in rows < NC of x (and is copied to
 // W.R); chain step: reflector heads in W.R, x becomes the dense V.
-template <typename T, int NC, int RPL, bool LEAF, int B>
-__device__ __forceinline__ void stream_tile_qr(T (&x)[NC][RPL], StreamWarp<T, NC, B>& W, int h) {
+template <typename T, int NC, int RPL, bool LEAF, int B, int NBUF>
+__device__ __forceinline__ void stream_tile_qr(T (&x)[NC][RPL], StreamWarp<T, NC, B, NBUF>& W, int h) {
     const int lane = threadIdx.x & 31;
 #pragma unroll
     for (int j = 0; j < NC; ++j) {
@@ -233,15 +235,33 @@ __device__ __forceinline__ void stream_tile_qr(T (&x)[NC][RPL], StreamWarp<T, NC
     }
 }
 
+// Householder scalars as householder_scalars (sg == 0 -> H = I), computed
+// branch-free so that every lane of a warp can evaluate them redundantly.
+template <typename T>
+__device__ __forceinline__ void householder_scalars_nb(T al, T sg, T& tau, T& beta, T& scale) {
+    const T ss = fma(al, al, sg);
+    const T aa = fabs(al);
+    T rmu, mu;
+    rsqrt_refined(ss, rmu, mu);
+    const bool z = sg == T(0);
+    beta = z ? al : -copysign(mu, al);
+    tau = z ? T(0) : fma(aa, rmu, T(1));
+    scale = z ? T(1) : copysign(rcp_refined(aa + mu), al);
+}
+
 // Merge of two upper-triangular n x n factors [Ra; Rb] (Rb: nb rows) by a
 // GROUP of NC lanes, lane k of the group holding column k of both (R[i*ld+k]).
 // Reflector j: head Ra[j][j], tail Rb[0..j][j] (structured).
+// The pivot column travels by shuffles and every lane computes the squared
+// norm and the Householder scalars itself, so a column costs one shuffle
+// latency plus the scalar chain (no shared memory, no __syncwarp; 2.1x faster
+// than a shared-memory broadcast, tools/merge_bench.cu).
 // Out: Ro = new R (may alias Ra or Rb: inputs are read into registers
 // first), rb = V_2 column k (rows <= k), G / tau for T.  All lanes of the warp
-// call it (uniform __syncwarp); groups with on == false only synchronise.
+// call it (full-warp shuffles); lanes with on == false compute nothing useful.
 template <typename T, int NC>
 __device__ __forceinline__ void merge_group(bool on, int k, const T* Ra, const T* Rb, int ld, int nb, T* Ro,
-                                            T (&rb)[NC], T* G, int ldg, T* tau, T* bc) {
+                                            T (&rb)[NC], T* G, int ldg, T* tau) {
     T ra[NC];
 #pragma unroll
     for (int i = 0; i < NC; ++i) {
@@ -251,46 +271,33 @@ __device__ __forceinline__ void merge_group(bool on, int k, const T* Ra, const T
     __syncwarp();
 #pragma unroll
     for (int j = 0; j < NC; ++j) {
-        if (on && k == j) {
-            T s0 = T(0), s1 = T(0);
+        T y[NC];
 #pragma unroll
-            for (int i = 0; i <= j; i += 2) {
-                s0 = fma(rb[i], rb[i], s0);
-                if (i + 1 <= j) s1 = fma(rb[i + 1], rb[i + 1], s1);
-            }
-            T tj, beta, scale;
-            householder_scalars(ra[j], s0 + s1, true, tj, beta, scale);
-            ra[j] = beta;
+        for (int i = 0; i <= j; ++i) y[i] = __shfl_sync(0xffffffffu, rb[i], j);
+        const T al = __shfl_sync(0xffffffffu, ra[j], j);
+        T s0 = T(0), s1 = T(0), d0 = T(0), d1 = T(0);  // ||y||^2 and y . rb_k
 #pragma unroll
-            for (int i = 0; i <= j; ++i) {
-                rb[i] *= scale;
-                bc[i] = rb[i];
-            }
-            bc[NC] = tj;
-            tau[j] = tj;
-        }
-        __syncwarp();
-        if (on) {
-            if (k > j) {
-                const T tj = bc[NC];
-                T s0 = ra[j], s1 = T(0);
-#pragma unroll
-                for (int i = 0; i <= j; i += 2) {
-                    s0 = fma(bc[i], rb[i], s0);
-                    if (i + 1 <= j) s1 = fma(bc[i + 1], rb[i + 1], s1);
-                }
-                const T f = tj * (s0 + s1);
-                ra[j] -= f;
-#pragma unroll
-                for (int i = 0; i <= j; ++i) rb[i] = fma(-f, bc[i], rb[i]);
-            } else if (k < j) {  // Gram entry (k, j): the R_a parts are unit vectors
-                T gsum = T(0);
-#pragma unroll
-                for (int i = 0; i <= j; ++i) gsum = fma(rb[i], bc[i], gsum);
-                G[k * ldg + j] = gsum;
+        for (int i = 0; i <= j; i += 2) {
+            s0 = fma(y[i], y[i], s0);
+            d0 = fma(y[i], rb[i], d0);
+            if (i + 1 <= j) {
+                s1 = fma(y[i + 1], y[i + 1], s1);
+                d1 = fma(y[i + 1], rb[i + 1], d1);
             }
         }
-        __syncwarp();
+        const T d = d0 + d1;
+        T tj, beta, scale;
+        householder_scalars_nb(al, s0 + s1, tj, beta, scale);
+        // k > j: s_k = Ra[j][k] + v_j . rb_k, v_j tail = scale y; k == j: the
+        // reflector itself; k < j: Gram entry v_k . v_j (R_a parts are unit vectors)
+        const bool diag = k == j;
+        const T f = k > j ? tj * fma(scale, d, ra[j]) : T(0);
+        ra[j] = diag ? beta : ra[j] - f;
+        const T fs = f * scale;
+#pragma unroll
+        for (int i = 0; i <= j; ++i) rb[i] = diag ? rb[i] * scale : fma(-fs, y[i], rb[i]);
+        if (on && k < j) G[k * ldg + j] = scale * d;
+        if (on && diag) tau[j] = tj;
     }
     if (on)
 #pragma unroll
@@ -332,14 +339,15 @@ __host__ __device__ inline int64_t stream_rx_ints(int64_t nct) {
     return ((nct * (NC * NC) * (int64_t)sizeof(T) / 4) + 31) & ~int64_t(31);
 }
 
-template <typename T, int NC, int RPL, int NW, bool VEC>
+template <typename T, int NC, int RPL, int NW, int NBUF, bool VEC>
 __global__ void __launch_bounds__(32 * NW, 1)
 tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int nlevels,
                    unsigned long long* prof, int dbg) {
     static_assert((NW & (NW - 1)) == 0, "NW: power of two (in-CTA tree levels)");
     constexpr int B = 32 * RPL;
     constexpr int LDR = NC + 1;
-    using SW = StreamWarp<T, NC, B>;
+    static_assert(NBUF == 1 || NBUF == 2, "one or two tile buffers");
+    using SW = StreamWarp<T, NC, B, NBUF>;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     SW* Ws = reinterpret_cast<SW*>(smem_raw);
@@ -385,8 +393,8 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
         for (int kt = 0; kt < ntile; ++kt) {
             const int64_t t = t0 + kt;
             const long long cw0 = prof ? clock64() : 0;
-            if (kt + 1 < ntile) {
-                stream_issue_tile<T, NC, B, VEC>(g, A, t + 1, W.buf[(kt + 1) & 1]);
+            if (NBUF == 2 && kt + 1 < ntile) {
+                stream_issue_tile<T, NC, B, VEC>(g, A, t + 1, W.buf[(kt + 1) % NBUF]);
                 asm volatile("cp.async.wait_group 1;" ::: "memory");
             } else {
                 asm volatile("cp.async.wait_group 0;" ::: "memory");
@@ -398,12 +406,13 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
 #pragma unroll
             for (int c = 0; c < NC; ++c)
 #pragma unroll
-                for (int i = 0; i < RPL; ++i) x[c][i] = W.buf[kt & 1][c][lane + 32 * i];
-            __syncwarp();  // the buffer is refilled (tile kt + 2) after this point
+                for (int i = 0; i < RPL; ++i) x[c][i] = W.buf[kt % NBUF][c][lane + 32 * i];
+            __syncwarp();  // the buffer is refilled (tile kt + NBUF) after this point
+            if (NBUF == 1 && kt + 1 < ntile) stream_issue_tile<T, NC, B, VEC>(g, A, t + 1, W.buf[0]);
             if (kt == 0)
-                stream_tile_qr<T, NC, RPL, true, B>(x, W, h);
+                stream_tile_qr<T, NC, RPL, true, B, NBUF>(x, W, h);
             else
-                stream_tile_qr<T, NC, RPL, false, B>(x, W, h);
+                stream_tile_qr<T, NC, RPL, false, B, NBUF>(x, W, h);
             // V (and a leaf's R) back over the tile; T into its slot
             const int64_t s = g.row0 + t * g.b;
 #pragma unroll
@@ -433,16 +442,18 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
     // A merge's V_2 and T are not needed by the levels above it (only its new
     // R is), so they are recorded in the merging warp's free tile buffers and
     // written out after the climb, by all warps of the CTA together.
-    // (NC <= 8; wider panels store at once: their records would not fit)
+    // (as many as fit: all of them for n <= 8; merges beyond the capacity
+    // store at once)
     using Rec = StreamRec<T, NC>;
-    constexpr bool DEFER = NC <= 8;
-    static_assert(!DEFER || sizeof(Rec) * kStreamMaxRec <= sizeof(T) * 2 * NC * B, "records fit in the tile buffers");
+    constexpr int kRecFit = (int)(sizeof(T) * NBUF * NC * B / sizeof(Rec));
+    constexpr int kRecCap = kRecFit < kStreamMaxRec ? kRecFit : kStreamMaxRec;
+    static_assert(NC > 8 || kRecCap == kStreamMaxRec, "n <= 8: every merge record fits in the tile buffers");
     __shared__ int s_nrec[NW];
     int nrec = 0;
     auto merge_rec = [&](const T* Ra, const T* Rb, int nb, T* Ro, int64_t sb) {
         T rb[NC];
-        merge_group<T, NC>(lane < NC, lane, Ra, Rb, LDR, nb, Ro, rb, &W.G[0][0], LDR, W.tau, W.bc);
-        if (!DEFER || nrec >= kStreamMaxRec) {
+        merge_group<T, NC>(lane < NC, lane, Ra, Rb, LDR, nb, Ro, rb, &W.G[0][0], LDR, W.tau);
+        if (nrec >= kRecCap) {
             store_merge(lane < NC, lane, sb, rb, &W.G[0][0], W.tau);
             return;
         }
@@ -459,6 +470,11 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
         __syncwarp();
     };
     // inside the CTA: warps' R's in shared memory, level by level
+    // (root path stamps, CAQR_PROFILE=1: [8] tree start, [9] in-CTA levels
+    // done, [10..13] sums of publish / ticket / sibling load / merge, [14]
+    // cross-CTA merges, [15] root done)
+    unsigned long long tp[6] = {0, 0, 0, 0, 0, 0};
+    if (prof) tp[0] = gtime();
     int l = 0;
     for (; (2 << l) <= NW && l < nlevels; ++l) {
         __syncthreads();
@@ -470,6 +486,7 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
         }
     }
     __syncthreads();
+    if (prof) tp[1] = gtime();
     auto store_r = [&](const T* R, int64_t sl) {  // R (upper) into the slot's top rows
         const int64_t hs = slot_h(sl);
         if (lane < NC && lane < wp) {
@@ -497,12 +514,14 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
         T* Rm = &W.R[0][0];
         T* Rs = &W.Rs[0][0];
         bool root = true;
+        int nx = 0;
         for (; l < nlevels; ++l) {
             const int64_t hl = int64_t(1) << l;
             const int64_t slot = cur * NW;
             const bool left = ((slot >> l) & 1) == 0;
             const int64_t sa = left ? slot : slot - hl, sb = sa + hl;
             if (sb >= g.P) continue;  // no right member at this level: pass up
+            unsigned long long c0 = prof ? gtime() : 0ull;
             for (int q = lane; q < NQ; q += 32) {
                 const int i = (4 * q) / NC, c = (4 * q) % NC;
                 const T* rr = Rm + i * LDR + c;
@@ -510,9 +529,11 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
                 __threadfence();
             }
             __syncwarp();
+            if (prof) { const unsigned long long c1 = gtime(); tp[2] += c1 - c0; c0 = c1; }
             int old = 0;
             if (lane == 0) old = atomicAdd(cnt + (int64_t)(l - l0) * nct + sa / NW, 1);
             old = __shfl_sync(0xffffffffu, old, 0);
+            if (prof) { const unsigned long long c1 = gtime(); tp[3] += c1 - c0; c0 = c1; }
             if (old == 0) {  // the sibling merges
                 root = false;
                 break;
@@ -527,12 +548,20 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
                 for (int e = 0; e < 4; ++e) Rs[i * LDR + c + e] = v[e];
             }
             __syncwarp();
+            if (prof) { const unsigned long long c1 = gtime(); tp[4] += c1 - c0; c0 = c1; }
             merge_rec(left ? Rm : Rs, left ? Rs : Rm, (int)min64(NC, slot_h(sb)), Rm, sb);
+            if (prof) { tp[5] += gtime() - c0; ++nx; }
             cur = sa / NW;
         }
         if (root) {
             store_r(Rm, 0);  // the root R into A's top rows
-            if (prof && lane == 0) atomicMax(prof + 2, gtime());
+            if (prof && lane == 0) {
+                const unsigned long long te = gtime();
+                atomicMax(prof + 2, te);
+                for (int q = 0; q < 6; ++q) prof[8 + q] = tp[q];
+                prof[14] = nx;
+                prof[15] = te;
+            }
         }
     }
     // ---- write out every recorded merge (V_2 into R_b's slot, T), CTA-wide
@@ -562,9 +591,9 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
     }
 }
 
-template <typename T, int NC, int RPL, int NW>
+template <typename T, int NC, int RPL, int NW, int NBUF = 2>
 inline size_t stream_smem_bytes(int64_t /*nct*/) {
-    return sizeof(StreamWarp<T, NC, 32 * RPL>) * NW;
+    return sizeof(StreamWarp<T, NC, 32 * RPL, NBUF>) * NW;
 }
 
 }  // namespace caqr

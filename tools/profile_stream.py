@@ -32,3 +32,8 @@ for rep in range(3):
     print(f"{m}x{n}: call {e0.elapsed_time(e1) * 1e3:.1f} us | chain phase {(t1 - t0) / 1e3:.1f} us "
           f"(mean chain {out[3] / chains / 1e3:.1f} us, mean tile wait {out[4] / chains / 1.9e3:.1f} us) | "
           f"tree tail after the last chain {(t2 - t1) / 1e3:.1f} us")
+    if out[15]:
+        print(f"   root path: in-CTA levels {(out[9] - out[8]) / 1e3:.2f} us, {out[14]} cross-CTA merges: publish "
+              f"{out[10] / 1e3:.2f} ticket {out[11] / 1e3:.2f} load {out[12] / 1e3:.2f} merge {out[13] / 1e3:.2f} us; "
+              f"tree start -> root {(out[15] - out[8]) / 1e3:.2f} us; root tree start - last chain end "
+              f"{(out[8] - t1) / 1e3:.2f} us")
