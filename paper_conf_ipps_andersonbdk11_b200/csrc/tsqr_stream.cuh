@@ -22,6 +22,7 @@
 //     CTA arrives SECOND at a pair (arrival counter) -- no one spins on a flag.
 #pragma once
 #include "tsqr_fused.cuh"
+#include "umma.cuh"
 
 namespace caqr {
 
@@ -84,6 +85,7 @@ __device__ __forceinline__ void householder_scalars(T al, T sg, bool live, T& ta
 template <typename T, int NC, int B, int NBUF = 2>
 struct alignas(16) StreamWarp {
     T buf[NBUF][NC][B];  // tile buffer(s) (column-major, B rows)
+    uint64_t mbar[2];  // bulk-copy completion, one per buffer
     T R[NC][NC + 1];   // chain / subtree R, R[j][k] (upper)
     T G[NC][NC + 1];   // Gram entries G[a][j] = v_a^T v_j (a < j)
     T Rs[NC][NC + 1];  // a sibling CTA's R (cross-CTA merges)
@@ -153,8 +155,35 @@ __device__ __forceinline__ void stream_issue_tile(const Geom& g, const T* A, int
     asm volatile("cp.async.commit_group;" ::: "memory");
 }
 
-// Leaf (kt == 0) or chain step (kt > 0) on the registers x[c][i] = row
-// lane + 32 i of column c.  Leaf: R ends in rows < NC of x (and is copied to
+// A full tile (B rows, 16-byte aligned columns) by the bulk-copy engine:
+// lane 0 posts the byte count on the buffer's mbarrier and issues one
+// column-sized copy per panel column (columns >= wp of the buffer stay zero).
+template <typename T, int NC, int B>
+__device__ __forceinline__ void stream_issue_bulk(const Geom& g, const T* A, int64_t t, T (*buf)[B],
+                                                  uint64_t* mbar) {
+    if ((threadIdx.x & 31) == 0) {
+        const int wp = g.ncols;
+        constexpr unsigned kBytes = B * sizeof(T);
+        const unsigned mb = umma::smem_u32(mbar);
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(kBytes * wp)
+                     : "memory");
+        const T* src = A + g.col0 * g.lda + g.row0 + t * g.b;
+        for (int c = 0; c < wp; ++c, src += g.lda)
+            asm volatile(
+                "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                    umma::smem_u32(&buf[c][0])),
+                "l"(src), "r"(kBytes), "r"(mb)
+                : "memory");
+    }
+}
+
+// Register layout of a tile: x[c][i] = row 128 (i / 4) + 4 lane + i % 4 of
+// column c, so a lane moves 16-byte pieces (LDS.128 from the tile buffer,
+// STG.128 of V).  Rows < 16 (R's rows) sit in lanes 0..3, i < 4.
+__device__ __forceinline__ int stream_row(int lane, int i) { return 128 * (i >> 2) + 4 * lane + (i & 3); }
+
+// Leaf (kt == 0) or chain step (kt > 0) on the registers x[c][i] (row
+// stream_row(lane, i) of column c).  Leaf: R ends in rows < NC of x (and is copied to
 // W.R); chain step: reflector heads in W.R, x becomes the dense V.
 template <typename T, int NC, int RPL, bool LEAF, int B, int NBUF>
 __device__ __forceinline__ void stream_tile_qr(T (&x)[NC][RPL], StreamWarp<T, NC, B, NBUF>& W, int h) {
@@ -167,7 +196,7 @@ __device__ __forceinline__ void stream_tile_qr(T (&x)[NC][RPL], StreamWarp<T, NC
         for (int q = 0; q < NC; ++q) red[q] = T(0);
 #pragma unroll
         for (int i = 0; i < RPL; ++i) {
-            const T xj = (LEAF && i == 0 && lane <= j) ? T(0) : x[j][i];
+            const T xj = (LEAF && i < 4 && 4 * lane + i <= j) ? T(0) : x[j][i];
             red[0] = fma(xj, xj, red[0]);
 #pragma unroll
             for (int q = 1; q < NC; ++q) {
@@ -182,7 +211,7 @@ __device__ __forceinline__ void stream_tile_qr(T (&x)[NC][RPL], StreamWarp<T, NC
 #pragma unroll
         for (int k = 0; k < NC; ++k) {
             if constexpr (LEAF)
-                hd[k] = __shfl_sync(0xffffffffu, x[k][0], j);
+                hd[k] = __shfl_sync(0xffffffffu, x[k][j & 3], j >> 2);
             else
                 hd[k] = k >= j ? W.R[j][k] : T(0);
         }
@@ -201,11 +230,12 @@ __device__ __forceinline__ void stream_tile_qr(T (&x)[NC][RPL], StreamWarp<T, NC
                 const T fs = f * scale;
 #pragma unroll
                 for (int i = 0; i < RPL; ++i) {
-                    if (LEAF && i == 0 && lane < j) continue;
-                    if (LEAF && i == 0 && lane == j)
-                        x[k][0] -= f;
-                    else
+                    if (LEAF && i < 4) {  // rows above the head keep, the head row takes -f
+                        const int r = 4 * lane + i;
+                        x[k][i] = r < j ? x[k][i] : (r == j ? x[k][i] - f : fma(-fs, x[j][i], x[k][i]));
+                    } else {
                         x[k][i] = fma(-fs, x[j][i], x[k][i]);
+                    }
                 }
                 if (!LEAF && lane == 0) W.R[j][k] = head - f;
             } else if (lane == 0) {  // Gram entry (a, j), a < j
@@ -215,11 +245,12 @@ __device__ __forceinline__ void stream_tile_qr(T (&x)[NC][RPL], StreamWarp<T, NC
         }
 #pragma unroll
         for (int i = 0; i < RPL; ++i) {
-            if (LEAF && i == 0 && lane < j) continue;
-            if (LEAF && i == 0 && lane == j)
-                x[j][0] = beta;
-            else
+            if (LEAF && i < 4) {
+                const int r = 4 * lane + i;
+                x[j][i] = r < j ? x[j][i] : (r == j ? beta : x[j][i] * scale);
+            } else {
                 x[j][i] *= scale;
+            }
         }
         if (lane == 0) {
             W.tau[j] = tau;
@@ -228,9 +259,13 @@ __device__ __forceinline__ void stream_tile_qr(T (&x)[NC][RPL], StreamWarp<T, NC
         __syncwarp();
     }
     if constexpr (LEAF) {  // R = rows < NC of the tile (upper part)
-        if (lane < NC)
 #pragma unroll
-            for (int k = 0; k < NC; ++k) W.R[lane][k] = k >= lane ? x[k][0] : T(0);
+        for (int e = 0; e < 4; ++e) {
+            const int r = 4 * lane + e;
+            if (r < NC)
+#pragma unroll
+                for (int k = 0; k < NC; ++k) W.R[r][k] = k >= r ? x[k][e] : T(0);
+        }
         __syncwarp();
     }
 }
@@ -347,6 +382,7 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
     constexpr int B = 32 * RPL;
     constexpr int LDR = NC + 1;
     static_assert(NBUF == 1 || NBUF == 2, "one or two tile buffers");
+    static_assert(RPL % 4 == 0, "rows move in 16-byte pieces (stream_row)");
     using SW = StreamWarp<T, NC, B, NBUF>;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -359,6 +395,11 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
     // condition compiles every shuffle to slow WARPSYNC.COLLECTIVE code)
     const bool live = __shfl_sync(0xffffffffu, chain < g.P ? 1 : 0, 0) != 0;
     const int wp = g.ncols;
+    // arrival counters of the in-CTA tree levels ([level][leftmost warp])
+    constexpr int kInLevels = NW >= 16 ? 4 : NW >= 8 ? 3 : NW >= 4 ? 2 : 1;
+    __shared__ int s_cnt[kInLevels * NW];
+    for (int i = threadIdx.x; i < kInLevels * NW; i += 32 * NW) s_cnt[i] = 0;
+    __syncthreads();
 
     // optional timestamps (diagnostics, CAQR_PROFILE=1): [0] min chain start,
     // [1] max chain end, [2] root done (ns, globaltimer); [3] sum of chain
@@ -389,16 +430,37 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
     if (live) {
         const int64_t t0 = chain * g.K;
         const int ntile = __shfl_sync(0xffffffffu, (int)min64(g.K, g.L - t0), 0);
-        stream_issue_tile<T, NC, B, VEC>(g, A, t0, W.buf[0]);
+        // Full tiles of a 16-byte aligned panel come by bulk copy (mbarrier
+        // per buffer), the rest -- a ragged last tile, or every tile of an
+        // unaligned panel -- by cp.async with zero fill.  Only the matrix's
+        // last tile (the last of its chain) can be ragged, so the bulk tiles
+        // of a buffer are consecutive uses and the wait parity is kt / NBUF.
+        auto bulk = [&](int64_t t) { return VEC && (t + 1) * g.b <= g.mrows; };
+        auto issue = [&](int64_t t, int bi) {
+            if (bulk(t))
+                stream_issue_bulk<T, NC, B>(g, A, t, W.buf[bi], &W.mbar[bi]);
+            else
+                stream_issue_tile<T, NC, B, VEC>(g, A, t, W.buf[bi]);
+        };
+        if (VEC) {
+            if (lane == 0)
+                for (int bi = 0; bi < NBUF; ++bi) umma::mbar_init(&W.mbar[bi], 1);
+            for (int bi = 0; bi < NBUF; ++bi)  // columns no bulk copy writes
+                for (int c = wp; c < NC; ++c)
+                    for (int r = lane; r < B; r += 32) W.buf[bi][c][r] = T(0);
+            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+            umma::fence_async_smem();
+            __syncwarp();
+        }
+        issue(t0, 0);
         for (int kt = 0; kt < ntile; ++kt) {
             const int64_t t = t0 + kt;
             const long long cw0 = prof ? clock64() : 0;
-            if (NBUF == 2 && kt + 1 < ntile) {
-                stream_issue_tile<T, NC, B, VEC>(g, A, t + 1, W.buf[(kt + 1) % NBUF]);
-                asm volatile("cp.async.wait_group 1;" ::: "memory");
-            } else {
+            if (NBUF == 2 && kt + 1 < ntile) issue(t + 1, (kt + 1) % NBUF);
+            if (bulk(t))
+                umma::mbar_wait(&W.mbar[kt % NBUF], (uint32_t)((kt / NBUF) & 1));
+            else
                 asm volatile("cp.async.wait_group 0;" ::: "memory");
-            }
             if (prof) twait += clock64() - cw0;
             __syncwarp();
             const int h = (int)min64(g.b, g.mrows - t * g.b);
@@ -406,9 +468,18 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
 #pragma unroll
             for (int c = 0; c < NC; ++c)
 #pragma unroll
-                for (int i = 0; i < RPL; ++i) x[c][i] = W.buf[kt % NBUF][c][lane + 32 * i];
+                for (int u = 0; u < RPL / 4; ++u) {
+                    const T* p = &W.buf[kt % NBUF][c][128 * u + 4 * lane];
+                    if constexpr (sizeof(T) == 4) {
+                        const float4 q = *reinterpret_cast<const float4*>(p);
+                        x[c][4 * u] = q.x, x[c][4 * u + 1] = q.y, x[c][4 * u + 2] = q.z, x[c][4 * u + 3] = q.w;
+                    } else {
+#pragma unroll
+                        for (int e = 0; e < 4; ++e) x[c][4 * u + e] = p[e];
+                    }
+                }
             __syncwarp();  // the buffer is refilled (tile kt + NBUF) after this point
-            if (NBUF == 1 && kt + 1 < ntile) stream_issue_tile<T, NC, B, VEC>(g, A, t + 1, W.buf[0]);
+            if (NBUF == 1 && kt + 1 < ntile) issue(t + 1, 0);
             if (kt == 0)
                 stream_tile_qr<T, NC, RPL, true, B, NBUF>(x, W, h);
             else
@@ -420,9 +491,15 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
                 if (c < wp) {
                     T* col = A + (g.col0 + c) * g.lda + s;
 #pragma unroll
-                    for (int i = 0; i < RPL; ++i) {
-                        const int r = lane + 32 * i;
-                        if (r < h) col[r] = x[c][i];
+                    for (int u = 0; u < RPL / 4; ++u) {
+                        const int r = 128 * u + 4 * lane;
+                        if (VEC && sizeof(T) == 4 && r + 4 <= h) {
+                            store_v4<T>(col + r, x[c][4 * u], x[c][4 * u + 1], x[c][4 * u + 2], x[c][4 * u + 3]);
+                        } else {
+#pragma unroll
+                            for (int e = 0; e < 4; ++e)
+                                if (r + e < h) col[r + e] = x[c][4 * u + e];
+                        }
                     }
                 }
             }
@@ -469,24 +546,18 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
         if (lane == 0) r.sb = sb;
         __syncwarp();
     };
-    // inside the CTA: warps' R's in shared memory, level by level
+    // The climb: every level's pair is merged by whichever member arrives
+    // SECOND (an arrival counter per pair; the first stops).  Inside the CTA
+    // a subtree's R lives in the shared R of the warp of its leftmost chain
+    // and the counters are shared-memory atomics; across CTAs the R travels
+    // through the workspace exchange area.  No barrier: the critical path is
+    // the last chain's own merges.  Release/acquire on the counters (one
+    // lane, after __syncwarp) publishes the R written by the whole warp.
     // (root path stamps, CAQR_PROFILE=1: [8] tree start, [9] in-CTA levels
     // done, [10..13] sums of publish / ticket / sibling load / merge, [14]
     // cross-CTA merges, [15] root done)
     unsigned long long tp[6] = {0, 0, 0, 0, 0, 0};
     if (prof) tp[0] = gtime();
-    int l = 0;
-    for (; (2 << l) <= NW && l < nlevels; ++l) {
-        __syncthreads();
-        const int hl = 1 << l;
-        const bool on = __shfl_sync(0xffffffffu, (live && (warp & (2 * hl - 1)) == 0 && chain + hl < g.P) ? 1 : 0, 0);
-        if (on) {  // warp-uniform
-            const int64_t sb = chain + hl;
-            merge_rec(&W.R[0][0], &Ws[warp + hl].R[0][0], (int)min64(NC, slot_h(sb)), &W.R[0][0], sb);
-        }
-    }
-    __syncthreads();
-    if (prof) tp[1] = gtime();
     auto store_r = [&](const T* R, int64_t sl) {  // R (upper) into the slot's top rows
         const int64_t hs = slot_h(sl);
         if (lane < NC && lane < wp) {
@@ -496,71 +567,119 @@ tsqr_stream_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, in
                 if (i <= lane && i < hs) col[i] = R[i * LDR + lane];
         }
     };
-    if (l >= nlevels) {  // the whole tree fitted in this CTA
-        if (warp == 0) store_r(&W.R[0][0], base);
-    } else if (warp == 0) {
-        // ---- across CTAs: the SECOND CTA to finish a pair merges it --------
-        // Same pairs, order and storage as a level-by-level tree, but no CTA
-        // waits: each publishes its R in the workspace exchange area and takes
-        // a ticket on the pair's arrival counter; the first arriver stops, the
-        // second merges [R_a; R_b] and climbs on.  Only lanes that write the
-        // R fence, so the publish does not wait for earlier V/T stores.
-        const int nct = (int)gridDim.x;
-        constexpr int NQ = NC * NC / 4;  // float4's per R
-        T* Rx = reinterpret_cast<T*>(sync + 64);          // [nct][NC][NC]
-        int* cnt = sync + 64 + stream_rx_ints<T, NC>(nct);  // [levels][nct]
-        const int l0 = l;
-        int64_t cur = blockIdx.x;  // CTA whose slot (cur * NW) this R belongs to
-        T* Rm = &W.R[0][0];
-        T* Rs = &W.Rs[0][0];
+    if (live) {
+        int64_t cur = chain;  // leftmost chain of this warp's subtree
         bool root = true;
-        int nx = 0;
-        for (; l < nlevels; ++l) {
-            const int64_t hl = int64_t(1) << l;
-            const int64_t slot = cur * NW;
-            const bool left = ((slot >> l) & 1) == 0;
-            const int64_t sa = left ? slot : slot - hl, sb = sa + hl;
+        int l = 0;
+        for (; (2 << l) <= NW && l < nlevels; ++l) {
+            const int hl = 1 << l;
+            const int64_t sa = cur & ~int64_t(2 * hl - 1), sb = sa + hl;
             if (sb >= g.P) continue;  // no right member at this level: pass up
-            unsigned long long c0 = prof ? gtime() : 0ull;
-            for (int q = lane; q < NQ; q += 32) {
-                const int i = (4 * q) / NC, c = (4 * q) % NC;
-                const T* rr = Rm + i * LDR + c;
-                store_v4<T>(Rx + cur * NC * NC + 4 * q, rr[0], rr[1], rr[2], rr[3]);
-                __threadfence();
-            }
             __syncwarp();
-            if (prof) { const unsigned long long c1 = gtime(); tp[2] += c1 - c0; c0 = c1; }
             int old = 0;
-            if (lane == 0) old = atomicAdd(cnt + (int64_t)(l - l0) * nct + sa / NW, 1);
+            if (lane == 0)
+                asm volatile("atom.acq_rel.cta.shared::cta.add.s32 %0, [%1], 1;"
+                             : "=r"(old)
+                             : "r"(umma::smem_u32(&s_cnt[l * NW + (int)(sa - base)]))
+                             : "memory");
             old = __shfl_sync(0xffffffffu, old, 0);
-            if (prof) { const unsigned long long c1 = gtime(); tp[3] += c1 - c0; c0 = c1; }
             if (old == 0) {  // the sibling merges
                 root = false;
                 break;
             }
-            __threadfence();
-            const int64_t other = (left ? sb : sa) / NW;
-            for (int q = lane; q < NQ; q += 32) {
-                const int i = (4 * q) / NC, c = (4 * q) % NC;
-                T v[4];
-                load_v4_cg<T>(Rx + other * NC * NC + 4 * q, v);
-#pragma unroll
-                for (int e = 0; e < 4; ++e) Rs[i * LDR + c + e] = v[e];
-            }
             __syncwarp();
-            if (prof) { const unsigned long long c1 = gtime(); tp[4] += c1 - c0; c0 = c1; }
-            merge_rec(left ? Rm : Rs, left ? Rs : Rm, (int)min64(NC, slot_h(sb)), Rm, sb);
-            if (prof) { tp[5] += gtime() - c0; ++nx; }
-            cur = sa / NW;
+            T* Ra = &Ws[sa - base].R[0][0];
+            merge_rec(Ra, &Ws[sb - base].R[0][0], (int)min64(NC, slot_h(sb)), Ra, sb);
+            cur = sa;
         }
-        if (root) {
-            store_r(Rm, 0);  // the root R into A's top rows
-            if (prof && lane == 0) {
-                const unsigned long long te = gtime();
-                atomicMax(prof + 2, te);
-                for (int q = 0; q < 6; ++q) prof[8 + q] = tp[q];
-                prof[14] = nx;
-                prof[15] = te;
+        if (prof) tp[1] = gtime();
+        if (root && l >= nlevels) {  // the whole tree fitted in this CTA
+            store_r(&Ws[0].R[0][0], base);
+        } else if (root) {
+            // ---- across CTAs -------------------------------------------------
+            const int nct = (int)gridDim.x;
+            constexpr int NQ = NC * NC / 4;  // float4's per R
+            T* Rx = reinterpret_cast<T*>(sync + 64);          // [nct][NC][NC]
+            int* cnt = sync + 64 + stream_rx_ints<T, NC>(nct);  // [levels][nct]
+            const int l0 = l;
+            int64_t cc = blockIdx.x;  // CTA whose slot (cc * NW) this R belongs to
+            T* Rm = &Ws[0].R[0][0];
+            T* Rs = &W.Rs[0][0];
+            int nx = 0;
+            // Poll every level above at once (lane q: level l0 + q, acquire):
+            // where the sibling subtree has already arrived, this CTA is the
+            // second at that pair whatever happens below, so it merges there
+            // without publishing its R or taking a ticket.  (The last CTA to
+            // finish finds all its siblings done: one round trip for the poll
+            // instead of a publish + ticket per level.)
+            unsigned ready = 0;
+            {
+                int v = 0;
+                const int lq = l0 + lane;
+                if (lq < nlevels && lq < 31) {
+                    const int64_t hl = int64_t(1) << lq;
+                    const int64_t sa = base & ~(2 * hl - 1), sb = sa + hl;
+                    if (sb < g.P)
+                        asm volatile("ld.acquire.gpu.global.s32 %0, [%1];"
+                                     : "=r"(v)
+                                     : "l"(cnt + (int64_t)(lq - l0) * nct + sa / NW)
+                                     : "memory");
+                }
+                ready = __ballot_sync(0xffffffffu, v != 0);
+                __syncwarp();
+            }
+            for (; l < nlevels; ++l) {
+                const int64_t hl = int64_t(1) << l;
+                const int64_t slot = cc * NW;
+                const bool left = ((slot >> l) & 1) == 0;
+                const int64_t sa = left ? slot : slot - hl, sb = sa + hl;
+                if (sb >= g.P) continue;  // no right member at this level: pass up
+                unsigned long long c0 = prof ? gtime() : 0ull;
+                if (!((ready >> (l - l0)) & 1u)) {  // publish, then the ticket decides
+                    for (int q = lane; q < NQ; q += 32) {
+                        const int i = (4 * q) / NC, c = (4 * q) % NC;
+                        const T* rr = Rm + i * LDR + c;
+                        store_v4<T>(Rx + cc * NC * NC + 4 * q, rr[0], rr[1], rr[2], rr[3]);
+                    }
+                    __syncwarp();
+                    if (prof) { const unsigned long long c1 = gtime(); tp[2] += c1 - c0; c0 = c1; }
+                    int old = 0;
+                    if (lane == 0)
+                        asm volatile("atom.acq_rel.gpu.global.add.s32 %0, [%1], 1;"
+                                     : "=r"(old)
+                                     : "l"(cnt + (int64_t)(l - l0) * nct + sa / NW)
+                                     : "memory");
+                    old = __shfl_sync(0xffffffffu, old, 0);
+                    if (prof) { const unsigned long long c1 = gtime(); tp[3] += c1 - c0; c0 = c1; }
+                    if (old == 0) {  // the sibling merges
+                        root = false;
+                        break;
+                    }
+                }
+                __syncwarp();
+                const int64_t other = (left ? sb : sa) / NW;
+                for (int q = lane; q < NQ; q += 32) {
+                    const int i = (4 * q) / NC, c = (4 * q) % NC;
+                    T v[4];
+                    load_v4_cg<T>(Rx + other * NC * NC + 4 * q, v);
+#pragma unroll
+                    for (int e = 0; e < 4; ++e) Rs[i * LDR + c + e] = v[e];
+                }
+                __syncwarp();
+                if (prof) { const unsigned long long c1 = gtime(); tp[4] += c1 - c0; c0 = c1; }
+                merge_rec(left ? Rm : Rs, left ? Rs : Rm, (int)min64(NC, slot_h(sb)), Rm, sb);
+                if (prof) { tp[5] += gtime() - c0; ++nx; }
+                cc = sa / NW;
+            }
+            if (root) {
+                store_r(Rm, 0);  // the root R into A's top rows
+                if (prof && lane == 0) {
+                    const unsigned long long te = gtime();
+                    atomicMax(prof + 2, te);
+                    for (int q = 0; q < 6; ++q) prof[8 + q] = tp[q];
+                    prof[14] = nx;
+                    prof[15] = te;
+                }
             }
         }
     }
