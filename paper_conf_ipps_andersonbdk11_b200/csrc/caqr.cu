@@ -12,6 +12,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <mutex>
+#include <vector>
 
 #include "../../include/caqr.h"
 #include "tsqr_fused.cuh"
@@ -31,12 +32,12 @@ static thread_local int g_last_cuda_error = 0;
 enum KernelId { K_PANEL_FACTOR = 0, K_PANEL_UPDATE = 1, K_EXTRACT_R = 2, K_SET_IDENTITY = 3,
                 K_TSQR_FUSED = 4, K_TSQR_SKINNY = 5, K_SVD_SMALL = 6, K_SVT_CORE = 7, K_EMBED_TOP = 8,
                 K_RPCA_UPDATE = 9, K_RPCA_INIT = 10, K_ABSMAX = 11, K_CHAIN_UPDATE = 12, K_STREAM_APPLY = 13,
-                K_TRSM = 14, K_TSQR_CHAIN = 15, K_NUM = 16 };
+                K_TRSM = 14, K_TSQR_CHAIN = 15, K_APPLY_ALL = 16, K_NUM = 17 };
 static const char* const kKernelNames[K_NUM] = {"panel_factor", "panel_update", "extract_r", "set_identity",
                                                 "tsqr_fused",   "tsqr_skinny",  "svd_small", "svt_core",
                                                 "embed_top",    "rpca_update",  "rpca_init", "absmax",
                                                 "node_update",  "stream_apply", "trsm_upper",
-                                                "tsqr_chain"};
+                                                "tsqr_chain",   "node_update_all"};
 struct Trace {
     std::mutex mu;
     bool on = false;
@@ -369,6 +370,98 @@ static int launch_update(const Geom& G, const T* A, const T* Tws, int level, int
 static inline bool chain_apply_policy() {
     const char* e = getenv("CAQR_CHAIN_APPLY");
     return !(e && e[0] == '0');
+}
+
+// CAQR_APPLY_ALL=0: one launch per tree level (+ one for the chains) instead
+// of node_update_all_kernel's single launch per group.
+static inline bool apply_all_policy() {
+    const char* e = getenv("CAQR_APPLY_ALL");
+    return !(e && e[0] == '0');
+}
+
+// Q^T C / Q C of a group -- chains (do_leaves) and every tree level -- in one
+// persistent launch (node_update_all_kernel); the tasks of each phase are
+// node_update_kernel's grid.  *done = false when the group does not qualify.
+template <typename T>
+static int launch_node_update_all(const Geom& G, const T* A, const T* Tws, bool do_leaves, T* C, int64_t ldc,
+                                  int64_t cfirst, int64_t ccount, int trans, cudaStream_t s, bool* done) {
+    *done = false;
+    if (!apply_all_policy()) return 0;
+    *done = true;
+    if (ccount <= 0) return 0;
+    const int nl = tree_levels(G.P);
+    std::vector<int> order;
+    if (trans) {
+        if (do_leaves) order.push_back(-1);
+        for (int lv = 0; lv < nl; ++lv) order.push_back(lv);
+    } else {
+        for (int lv = nl - 1; lv >= 0; --lv) order.push_back(lv);
+        if (do_leaves) order.push_back(-1);
+    }
+    ApplyPhases ph{};
+    const int64_t nblk = ceil_div(ccount, 32);
+    int rgmax = 0;
+    double fl = 0, by = 0;
+    for (int level : order) {
+        const int64_t nodes = level < 0 ? G.P : merges_at(G.P, level);
+        if (nodes <= 0) continue;
+        if (ph.n >= kMaxApplyPhases) {
+            *done = false;
+            return 0;
+        }
+        const int64_t groups = std::max<int64_t>(1, std::min<int64_t>(nblk, (2 * num_sms()) / nodes));
+        const int64_t cpb = ceil_div(nblk, groups);
+        const int64_t gy = ceil_div(nblk, cpb);
+        if ((int64_t)ph.start[ph.n] + nodes * gy > INT32_MAX / 2) {
+            *done = false;
+            return 0;
+        }
+        ph.level[ph.n] = level;
+        ph.nodes[ph.n] = (int)nodes;
+        ph.cpb[ph.n] = (int)cpb;
+        ph.start[ph.n + 1] = ph.start[ph.n] + (int)(nodes * gy);
+        ++ph.n;
+        rgmax = std::max(rgmax, level < 0 ? (int)(G.K > 1 ? G.b + kPW : std::min<int64_t>(G.b, G.mrows))
+                                          : (int)(kPW + std::min<int64_t>(G.ncols, G.b)));
+        if (g_trace.on)
+            for (int kt = 0; kt < (level < 0 ? G.K : 1); ++kt)
+                for (int p = 0; p < G.npan; ++p) {
+                    double f1, b1;
+                    trace_counts(G, level, p, kt, nodes, true, ccount, sizeof(T), &f1, &b1);
+                    fl += f1;
+                    by += b1;
+                }
+    }
+    const int total = ph.start[ph.n];
+    if (total == 0) return 0;
+    const size_t smem = panel_update_smem<T>(rgmax);
+    cudaError_t e = allow_smem(node_update_all_kernel<T>, smem);
+    int occ = 0;  // a cooperative grid: every CTA resident
+    if (e == cudaSuccess)
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, node_update_all_kernel<T>, kThreads, smem);
+    if (e == cudaSuccess && occ < 1) {
+        *done = false;
+        return 0;
+    }
+    if (e == cudaSuccess) {
+        TraceScope ts(K_APPLY_ALL, fl, by, s);
+        const unsigned grid = (unsigned)std::min<int64_t>(total, (int64_t)occ * num_sms());
+        Geom g = G;
+        const T* a = A;
+        const T* tw = Tws;
+        T* c = C;
+        int64_t ld = ldc, cf = cfirst, cc = ccount;
+        int tr = trans;
+        void* args[] = {&g, &a, &tw, &c, &ld, &cf, &cc, &tr, &ph};
+        e = cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(node_update_all_kernel<T>), dim3(grid),
+                                        dim3(kThreads), args, smem, s);
+        if (e == cudaSuccess) e = cudaGetLastError();
+    }
+    if (e != cudaSuccess) {
+        g_last_cuda_error = (int)e;
+        return CAQR_ERR_CUDA;
+    }
+    return 0;
 }
 
 template <typename T>
@@ -828,6 +921,21 @@ static int apply_group(const Geom& G, const T* A, const T* Tws, bool do_leaves, 
     int rc = 0;
     const int nl = tree_levels(G.P);
     if (!mma && chain_apply_policy()) {  // one launch per tree level (+ one for the chains)
+        // groups the warp-per-chain skinny apply does not take: one launch
+        const bool skinny = sizeof(T) == 4 && G.npan == 1 &&
+                            ((G.ncols <= 8 && G.b == 256) || (G.ncols <= 16 && G.b == 128));
+        if (!skinny || (getenv("CAQR_STREAM_APPLY") && getenv("CAQR_STREAM_APPLY")[0] == '0')) {
+            bool done = false;
+            const char* dbg = getenv("CAQR_APPLY_ALL");
+            if (dbg && dbg[0] == '2') {  // diagnostics: chains by node_update_kernel, tree in one launch
+                if (trans && do_leaves) rc = launch_node_update<T>(G, A, Tws, -1, C, ldc, cfirst, ccount, 1, s);
+                if (!rc) rc = launch_node_update_all<T>(G, A, Tws, false, C, ldc, cfirst, ccount, trans, s, &done);
+                if (!rc && !trans && do_leaves) rc = launch_node_update<T>(G, A, Tws, -1, C, ldc, cfirst, ccount, 0, s);
+                return rc;
+            }
+            rc = launch_node_update_all<T>(G, A, Tws, do_leaves, C, ldc, cfirst, ccount, trans, s, &done);
+            if (rc || done) return rc;
+        }
         auto leaves = [&](int tr) {
             bool done = false;
             int r = launch_stream_apply<T>(G, A, Tws, C, ldc, cfirst, ccount, tr, s, &done);

@@ -25,6 +25,7 @@
 // the sparsity pattern") and keep the leaves' vectors that share those rows
 // untouched (tree vectors overwrite exactly the R slots).
 #pragma once
+#include <cooperative_groups.h>
 #include <cstdint>
 #include <cuda_runtime.h>
 
@@ -632,6 +633,52 @@ node_update_kernel(Geom g, const T* A, const T* __restrict__ Tws, int level, T* 
         const int p = trans ? s % g.npan : g.npan - 1 - s % g.npan;
         update_node<T, MMA>(g, A, Tws, level, node, p, kt, C, ldc, cfirst, ccount, trans, blk_beg, blk_end,
                             smem_raw);
+    }
+}
+
+// Q^T C / Q C of a whole group in ONE launch (the device
+// steps through the tree levels instead of the host, cf. the early start of
+// P:L356-360).  The phases -- the chains (level -1) and the tree levels, in
+// execution order (bottom-up for Q^T, top-down for Q) -- are cut into tasks
+// (node, group of 32-column blocks) exactly as node_update_kernel's grid;
+// a cooperative grid of resident CTAs strides over each phase's tasks and
+// meets at a grid barrier between phases (no scratch memory: the apply calls
+// take the workspace read-only).  Each node runs the same update_node calls
+// in the same order as the per-level launches: the results are bitwise equal
+// (tests/test_gpu_parity.py).
+constexpr int kMaxApplyPhases = 40;
+struct ApplyPhases {
+    int n;                          // phases
+    int level[kMaxApplyPhases];     // -1: the chains
+    int nodes[kMaxApplyPhases];     // nodes of the phase
+    int cpb[kMaxApplyPhases];       // 32-column blocks per task
+    int start[kMaxApplyPhases + 1]; // first task of each phase (prefix sums)
+};
+
+template <typename T>
+__global__ void __launch_bounds__(kThreads, sizeof(T) == 4 ? 2 : 1)  // fp32: node_update_kernel's 2 CTAs/SM
+node_update_all_kernel(Geom g, const T* A, const T* __restrict__ Tws, T* C, int64_t ldc, int64_t cfirst,
+                       int64_t ccount, int trans, ApplyPhases ph) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    cooperative_groups::grid_group grid = cooperative_groups::this_grid();
+    const int64_t nblk = (ccount + 31) / 32;
+    for (int q = 0; q < ph.n; ++q) {
+        if (q > 0) grid.sync();  // phase q-1 done everywhere (and its C stores visible)
+        const int level = ph.level[q];
+        const int ntask = ph.start[q + 1] - ph.start[q];
+        for (int local = blockIdx.x; local < ntask; local += gridDim.x) {
+            const int64_t node = local % ph.nodes[q];
+            const int64_t blk_beg = (int64_t)(local / ph.nodes[q]) * ph.cpb[q];
+            const int64_t blk_end = min(nblk, blk_beg + ph.cpb[q]);
+            const int ntile = level < 0 ? (int)min(g.K, g.L - node * g.K) : 1;
+            const int steps = ntile * g.npan;
+            for (int s = 0; s < steps; ++s) {
+                const int kt = trans ? s / g.npan : ntile - 1 - s / g.npan;
+                const int p = trans ? s % g.npan : g.npan - 1 - s % g.npan;
+                update_node<T, false>(g, A, Tws, level, node, p, kt, C, ldc, cfirst, ccount, trans, blk_beg,
+                                      blk_end, smem_raw);
+            }
+        }
     }
 }
 

@@ -571,10 +571,43 @@ def test_node_update_matches_per_panel_launches(caqr, m, n, dtype, monkeypatch):
         return Q.cpu().numpy(), C.cpu().numpy(), D.cpu().numpy()
 
     new = run()
+    monkeypatch.setenv("CAQR_APPLY_ALL", "0")
+    per_level = run()
     monkeypatch.setenv("CAQR_CHAIN_APPLY", "0")
     old = run()
-    for a, b in zip(new, old):
+    for a, b, c in zip(new, per_level, old):
         assert np.array_equal(a, b)
+        assert np.array_equal(b, c)
+
+
+@pytest.mark.parametrize("m,n,dtype", [(1_000_000, 192, np.float32), (200_000, 100, np.float64)])
+def test_apply_one_launch_per_group(caqr, m, n, dtype):
+    """Q^T C and form_q of a one-group plan are ONE apply
+    launch (node_update_all_kernel schedules the chains and every tree level
+    on the device) -- counted from the launch trace."""
+    tdt = torch.float32 if dtype == np.float32 else torch.float64
+    Ad = workloads.device_gaussian(m, n, seed=3, dtype=tdt, device="cuda").t()
+    A = caqr.colmajor_empty(m, n, tdt)
+    A.copy_(Ad)
+    R, ws = caqr.caqr_factor(A)
+    info = caqr.caqr_plan_info(m, n, 0 if dtype == np.float32 else 1)
+    assert info["groups"] == 1 and info["tree_levels"] >= 5
+    C = caqr.colmajor(Ad[:, :4].clone())
+    torch.cuda.synchronize()
+    caqr.caqr_trace_begin(1 << 12)
+    caqr.caqr_apply_qt(A, ws, C)
+    Q = caqr.caqr_form_q(A, ws)
+    torch.cuda.synchronize()
+    names = [t[0] for t in caqr.caqr_trace_end(1 << 12)]
+    assert names.count("node_update_all") == 2, names
+    assert "node_update" not in names and "panel_update" not in names, names
+    # and the result is Q: Q^T Q = I, Q^T A = [R; 0] on the top rows
+    bd = BOUNDS[dtype]
+    Q64 = Q.double()
+    eye = torch.eye(n, dtype=torch.float64, device="cuda")
+    assert (Q64.t() @ Q64 - eye).norm().item() <= bd["orth"]
+    top = (Q64.t() @ Ad[:, :4].double() - C[:n].double()).norm() / Ad[:, :4].double().norm()
+    assert top.item() <= bd["res"]
 
 
 @pytest.mark.parametrize("m,n,k", [(4_000_000, 8, 8), (600_001, 5, 11), (1_000_003, 16, 16), (262_147, 12, 3)])
