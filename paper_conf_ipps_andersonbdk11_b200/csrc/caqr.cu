@@ -917,14 +917,14 @@ static int factor_group(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, 
 template <typename T>
 static int apply_group(const Geom& G, const T* A, const T* Tws, bool do_leaves, T* C,
                        int64_t ldc, int64_t cfirst, int64_t ccount, int trans, cudaStream_t s,
-                       bool mma = false) {
+                       bool mma = false, bool one_launch = true) {
     int rc = 0;
     const int nl = tree_levels(G.P);
     if (!mma && chain_apply_policy()) {  // one launch per tree level (+ one for the chains)
         // groups the warp-per-chain skinny apply does not take: one launch
         const bool skinny = sizeof(T) == 4 && G.npan == 1 &&
                             ((G.ncols <= 8 && G.b == 256) || (G.ncols <= 16 && G.b == 128));
-        if (!skinny || (getenv("CAQR_STREAM_APPLY") && getenv("CAQR_STREAM_APPLY")[0] == '0')) {
+        if (one_launch && (!skinny || (getenv("CAQR_STREAM_APPLY") && getenv("CAQR_STREAM_APPLY")[0] == '0'))) {
             bool done = false;
             const char* dbg = getenv("CAQR_APPLY_ALL");
             if (dbg && dbg[0] == '2') {  // diagnostics: chains by node_update_kernel, tree in one launch
@@ -1060,8 +1060,10 @@ static int factor_impl(int64_t m, int64_t n, T* A, int64_t lda, T* R, int64_t ld
             if (!rc && cudaEventRecord(ev_done, s2) != cudaSuccess) rc = CAQR_ERR_CUDA;
         }
         if (!rc && next_cols < n - trail0)
+            // (per-level launches: a cooperative grid would hold every SM and
+            // shut out the next TSQR running beside it on s2; C5 76 -> 95 ms)
             rc = apply_group<T>(G, A, Tws, true, A, lda, trail0 + next_cols, n - trail0 - next_cols, 1, s,
-                                mma_policy());
+                                mma_policy(), !overlap);
     }
     if (!rc) rc = launch_extract_r<T>(n, A, lda, R, ldr, s);
     return rc;
@@ -1589,11 +1591,17 @@ int caqr_plan_info(int64_t m, int64_t n, int dtype, const caqr_opts* opts, int64
     for (int64_t g = 0; g < pl.ngroups; ++g) {
         const Geom Gg = group_geom(pl, g, m);
         const int nl = tree_levels(Gg.P);
-        if (fused_ok(Gg) || (pl.skinny && Gg.npan == 1))
+        if (pl.chain)
+            launches += 2;  // chain kernel + the fused kernel's tree
+        else if (fused_ok(Gg) || (pl.skinny && Gg.npan == 1))
             launches += 1;
         else
             launches += (int64_t)(nl + Gg.K) * (2 * Gg.npan - 1);
-        if (Gg.col0 + Gg.ncols < n) launches += (int64_t)(nl + Gg.K) * Gg.npan;
+        const int64_t trail0 = Gg.col0 + Gg.ncols;
+        if (trail0 < n) {  // trailing update (defaults: early start, FFMA apply)
+            launches += 1;  // the next group's columns: one cooperative launch
+            if (n - trail0 > pl.nb) launches += nl + 1;  // the rest beside the next TSQR: chains + levels
+        }
     }
     out[6] = launches;
     return 0;

@@ -68,8 +68,8 @@ def test_plan_info(L):
     assert p["panel_cols"] == 64 and p["groups"] == 128
     p = caqr.caqr_plan_info(4096, 16, 0, caqr.make_opts(leaf_rows=128))
     assert p["leaf_rows"] == 128 and p["leaves"] == 32 and p["tree_levels"] == 5
-    p = caqr.caqr_plan_info(4_000_000, 8)  # skinny: 256-row tiles, ~2048 chains
-    assert p["leaf_rows"] == 256 and p["leaves"] == 15625 and p["chains"] == 1117 and p["launches"] == 2
+    p = caqr.caqr_plan_info(4_000_000, 8)  # skinny: 256-row tiles, ~2368 chains (16 warps x 148 SMs)
+    assert p["leaf_rows"] == 256 and p["leaves"] == 15625 and p["chains"] == 2233 and p["launches"] == 2
 
 
 def test_info_codes_without_gpu(L):
