@@ -298,7 +298,26 @@ def extra_configs_leg(args, dev, flush, peaks):
             flush.zero_()
 
         steps = min(args.steps, 5 if m * n > 5e7 else 20)
-        ms = timed_steps(lambda: caqr.caqr_factor(A, R=R, ws=ws, opts=opts), prep, args.warmup, steps, stream)
+        step = lambda: caqr.caqr_factor(A, R=R, ws=ws, opts=opts)  # noqa: E731
+        ms = timed_steps(step, prep, args.warmup, steps, stream)
+        # the same C-ABI call replayed from a CUDA graph: the device time
+        # without the ~25 us of host work per call (Python + ctypes + plan +
+        # launches), which dominates the small configs (C1, C2)
+        gms = None
+        try:
+            g = torch.cuda.CUDAGraph()
+            side = torch.cuda.Stream()
+            side.wait_stream(stream)
+            with torch.cuda.stream(side):
+                prep()
+                step()
+            stream.wait_stream(side)
+            with torch.cuda.graph(g):
+                step()
+            gms = timed_steps(g.replay, prep, args.warmup, steps, stream)
+            del g
+        except Exception as exc:  # noqa: BLE001 -- reported, the eager number stands
+            gms = f"graph capture failed: {exc}"
         fl = 2.0 * m * n * n - 2.0 * n ** 3 / 3.0
         alu = alu_peak_tflops(dt, peaks["sm_max_mhz"])
         t_roof = max(2.0 * m * n * esz / (peaks["hbm_gbs"] * 1e9), fl / (alu * 1e12))
@@ -306,7 +325,12 @@ def extra_configs_leg(args, dev, flush, peaks):
                      "read_write_gbs": 2.0 * m * n * esz / (ms * 1e-3) / 1e9,
                      "roofline_frac": t_roof / (ms * 1e-3),
                      "roofline_note": "max(read A + write V at measured HBM, flops at derived ALU peak) / time",
+                     "graph_ms_per_step": gms,
+                     "graph_note": "same caqr_factor call captured once and replayed (CUDA graph); "
+                                   "same prep / events protocol; excludes host launch cost",
                      "plan": caqr.caqr_plan_info(m, n, code, opts)}
+        if isinstance(gms, float):
+            out[name]["graph_roofline_frac"] = t_roof / (gms * 1e-3)
         del A0, A, R, ws
         torch.cuda.empty_cache()
     return out

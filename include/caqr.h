@@ -68,14 +68,16 @@ typedef struct CUstream_st *caqr_stream_t; /* == cudaStream_t */
 enum { CAQR_F32 = 0, CAQR_F64 = 1 };
 enum { CAQR_OK = 0, CAQR_ERR_CUDA = 1, CAQR_ERR_NCCL = 2, CAQR_ERR_UNSUPPORTED = 3, CAQR_ERR_TIMEOUT = 4 };
 
-/* Plan options; a field <= 0 means "default".
+/* Plan options; a field <= 0 means "default" (caqr_tune searches them).
  *   leaf_rows  b: rows per TSQR tile (P:L633 / P:L822-823 used 64 and 128 on
  *              Fermi; here a multiple of 32, b >= the panel-group width,
- *              b <= 256).  Default 224 (256 for groups wider than 224).
+ *              b <= 256).  Default 224 for n <= 224, 256 for wider matrices;
+ *              fp32 n <= 16 (streaming kernel): 256 for n <= 8, 128 for n <= 16.
  *              Consecutive tiles form chains (flat trees) of K = ceil(L/296)
- *              tiles; the chains' R factors are reduced by a binary tree.
+ *              tiles (skinny: ~1184 / 2368 chains); the chains' R factors are
+ *              reduced by a binary tree.
  *   panel_cols nb: CAQR panel-group width (one TSQR per group).
- *              Default: n if n <= 256 (one whole-width TSQR), else 64. */
+ *              Default: n if n <= 224 (one whole-width TSQR), else 128. */
 typedef struct caqr_opts {
     int64_t leaf_rows;
     int64_t panel_cols;
@@ -377,6 +379,27 @@ int caqr_debug_profile_read(unsigned long long out[16]);
  * tree_levels(group 0), panels(group 0), kernel_launches(factor), chains(group 0)}.
  * Returns 0 or a negative info. */
 int caqr_plan_info(int64_t m, int64_t n, int dtype, const caqr_opts *opts, int64_t out[8]);
+
+/* Plan search (the paper tunes its block sizes by search,
+ * P:L796-804 Sec. IV.F, and picks the algorithm by shape).
+ * Times caqr_factor of the m x n matrix A (device, column-major, lda; NOT
+ * modified: every trial factors a scratch copy) for each candidate plan --
+ * leaf_rows in {default, 64, 96, ..., 256} x panel_cols in {default, 32, 64,
+ * ..., 256} (< n), keeping only valid plans that differ in (tile height,
+ * group width, kernel family) -- as the median of `reps` (1..50) calls after
+ * one warm-up, CUDA events on `stream`.
+ *   best        out: the fastest plan's options (all-zero when the default
+ *               plan is fastest; ties keep the default)           (-7 if NULL)
+ *   best_ms     out: its time (ms)                                 (-7 if NULL)
+ *   default_ms  out (may be NULL): the default plan's time (ms)
+ *   ntried      out (may be NULL): plans timed
+ * Info: -1 m < 0, -2 n < 0 or n > m, -3 dtype, -4 A NULL, -5 lda < m; or a
+ * factor error; CAQR_ERR_CUDA.  Allocates its scratch (a copy of A, R, the
+ * largest workspace) with cudaMalloc and synchronises on `stream`: a setup
+ * call, not for graph capture.  Tested: tests/test_gpu_parity.py
+ * (test_tune_*). */
+int caqr_tune(int64_t m, int64_t n, int dtype, const void *A, int64_t lda, int reps, caqr_opts *best,
+              float *best_ms, float *default_ms, int *ntried, caqr_stream_t stream);
 
 #ifdef __cplusplus
 }

@@ -92,6 +92,9 @@ def lib() -> ctypes.CDLL:
         L.caqr_build_info.restype = ctypes.c_char_p
         L.caqr_plan_info.argtypes = [i64, i64, ip, op, ctypes.POINTER(ctypes.c_int64)]
         L.caqr_plan_info.restype = ip
+        L.caqr_tune.argtypes = [i64, i64, ip, vp, i64, ip, ctypes.POINTER(Opts), ctypes.POINTER(ctypes.c_float),
+                                ctypes.POINTER(ctypes.c_float), ctypes.POINTER(ip), vp]
+        L.caqr_tune.restype = ip
         L.caqr_trace_begin.argtypes = [ip]
         L.caqr_trace_begin.restype = ip
         L.caqr_trace_end.argtypes = [ctypes.POINTER(ip), ctypes.POINTER(ctypes.c_float),
@@ -222,6 +225,20 @@ def caqr_plan_info(m: int, n: int, dtype: int = CAQR_F32, opts: Optional[Opts] =
     _check("caqr_plan_info", lib().caqr_plan_info(m, n, dtype, _optp(opts), out))
     keys = ["leaf_rows", "panel_cols", "groups", "leaves", "tree_levels", "panels", "launches", "chains"]
     return {k: int(out[i]) for i, k in enumerate(keys)}
+
+
+def caqr_tune(A, reps: int = 3, stream=None):
+    """Plan search on the column-major CUDA matrix A (left unchanged).  Returns
+    (opts or None for the default plan, best_ms, default_ms, plans_tried)."""
+    code, _ = _dtype_code(A)
+    m, n = A.shape
+    pa, lda = _colmajor(A, "A")
+    best = Opts()
+    bms, dms, nt = ctypes.c_float(), ctypes.c_float(), ctypes.c_int()
+    _check("caqr_tune", lib().caqr_tune(m, n, code, pa, lda, reps, ctypes.byref(best), ctypes.byref(bms),
+                                        ctypes.byref(dms), ctypes.byref(nt), _stream(stream)))
+    opts = best if (best.leaf_rows or best.panel_cols) else None
+    return opts, float(bms.value), float(dms.value), int(nt.value)
 
 
 def caqr_factor(A, R=None, ws=None, opts: Optional[Opts] = None, stream=None):

@@ -117,8 +117,11 @@ static int make_plan(int64_t m, int64_t n, int dtype, const caqr_opts* o, int op
     // n in (224, 256] -- a 256-wide group's top tree merges need 2*32 + 224 =
     // 288 > 256 gathered rows, which only the per-level split path takes (SURVEY
     // 8(f) f3: 8192 x 256 was 6 ms that way, vs two 128-wide CAQR groups);
-    // 64-wide CAQR panels beyond
-    int64_t nb = (o && o->panel_cols > 0) ? o->panel_cols : (n <= 224 ? n : (n <= kMaxGroup ? 128 : 64));
+    // 128-wide CAQR groups beyond (round 2: caqr_tune's search put (b, nb) =
+    // (256, 128) first or within a few % on every wide shape measured --
+    // 8192^2 68.8 vs 75.6 ms for nb = 64, 4096^2 f64 29.0 vs 32.5 ms,
+    // profiles/round2_measurements.txt)
+    int64_t nb = (o && o->panel_cols > 0) ? o->panel_cols : (n <= 224 ? n : 128);
     if (nb > kMaxGroup) return -opt_pos;
     nb = std::max<int64_t>(1, std::min(nb, std::max<int64_t>(n, 1)));
     // skinny fp32 panels (n <= 16, one group): one warp per chain, 256-row (n <= 8)
@@ -145,7 +148,7 @@ static int make_plan(int64_t m, int64_t n, int dtype, const caqr_opts* o, int op
     int64_t b = (o && o->leaf_rows > 0) ? o->leaf_rows
                                         : pl->chain ? chain_tile_rows(n)
                                         : (pl->skinny ? (n <= 8 && !s16 ? 256 : 128)
-                                                      : (nb <= kFusedLeaf ? kFusedLeaf : kMaxLeaf));
+                                                      : (nb <= kFusedLeaf && n <= 224 ? kFusedLeaf : kMaxLeaf));
     if (b % 32 != 0 || b > kMaxLeaf) return -opt_pos;
     b = std::max(b, round_up(nb, 32));
     if (b > kMaxLeaf) return -opt_pos;
@@ -298,6 +301,35 @@ template <typename K>
 static cudaError_t allow_smem(K kernel, size_t bytes) {
     return allow_smem_ptr(reinterpret_cast<const void*>(kernel), bytes);
 }
+// Resident CTAs per SM of (kernel, threads, dynamic smem) on the current
+// device, cached (the runtime query costs tens of microseconds of host time
+// per call -- as much as a small factorisation's device time).
+static cudaError_t occupancy_ptr(int* occ, const void* kernel, int threads, size_t smem) {
+    struct Key {
+        const void* k;
+        int dev, threads;
+        size_t smem;
+        int occ;
+    };
+    static std::mutex mu;
+    static Key keys[256];
+    static int nkeys = 0;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    std::lock_guard<std::mutex> lk(mu);
+    for (int i = 0; i < nkeys; ++i)
+        if (keys[i].k == kernel && keys[i].dev == dev && keys[i].threads == threads && keys[i].smem == smem) {
+            *occ = keys[i].occ;
+            return cudaSuccess;
+        }
+    const cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, kernel, threads, smem);
+    if (e == cudaSuccess && nkeys < 256) keys[nkeys++] = Key{kernel, dev, threads, smem, *occ};
+    return e;
+}
+template <typename K>
+static cudaError_t occupancy(int* occ, K kernel, int threads, size_t smem) {
+    return occupancy_ptr(occ, reinterpret_cast<const void*>(kernel), threads, smem);
+}
 
 template <typename T>
 static int launch_factor(const Geom& G, T* A, T* Tws, int level, int p, int kt, int64_t nodes,
@@ -438,7 +470,7 @@ static int launch_node_update_all(const Geom& G, const T* A, const T* Tws, bool 
     cudaError_t e = allow_smem(node_update_all_kernel<T>, smem);
     int occ = 0;  // a cooperative grid: every CTA resident
     if (e == cudaSuccess)
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, node_update_all_kernel<T>, kThreads, smem);
+        e = occupancy(&occ, node_update_all_kernel<T>, kThreads, smem);
     if (e == cudaSuccess && occ < 1) {
         *done = false;
         return 0;
@@ -614,7 +646,7 @@ static int launch_fused(const Geom& G, T* A, T* Tws, int* sync, bool do_leaves, 
         if (e == cudaSuccess) e = allow_smem(tsqr_fused_kernel<T>, smem);
         int occ = 1;
         if (e == cudaSuccess)
-            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, tsqr_fused_kernel<T>, kThreads, smem);
+            e = occupancy(&occ, tsqr_fused_kernel<T>, kThreads, smem);
         if (e == cudaSuccess) {
             const int64_t grid = std::min<int64_t>(total, (int64_t)std::max(occ, 1) * num_sms());
             TraceScope ts(K_TSQR_FUSED, fl, by, s);
@@ -803,7 +835,7 @@ static cudaError_t launch_chain_cfg(const Geom& G, float* A, float* Tws, int* sy
     auto kern = tsqr_chain_kernel<NQ, SEG, MINB, TC>;
     cudaError_t e = allow_smem(kern, smem);
     int occ = 1;
-    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, 32 * NQ, smem);
+    if (e == cudaSuccess) e = occupancy(&occ, kern, 32 * NQ, smem);
     if (e != cudaSuccess) return e;
     if (TC) {
         // The occupancy API counts a tcgen05 kernel as one CTA per SM; the
@@ -1431,7 +1463,111 @@ static int factor_host_impl(int64_t m, int64_t n, int S, const T* Ah, int64_t ld
                            dtype);
 }
 
+// Plan search (caqr_tune): every candidate (leaf_rows, panel_cols) whose plan
+// is valid and distinct, timed on a scratch copy of A.
+template <typename T>
+static int tune_impl(int64_t m, int64_t n, const T* A, int64_t lda, int reps, int dtype, caqr_opts* best,
+                     float* best_ms, float* default_ms, int* ntried, cudaStream_t s) {
+    if (m < 0) return -1;
+    if (n < 0 || n > m) return -2;
+    if (lda < std::max<int64_t>(1, m)) return -5;
+    if (!best || !best_ms) return -7;
+    if (!A && m > 0 && n > 0) return -4;
+    *best = caqr_opts{};
+    *best_ms = 0.f;
+    if (default_ms) *default_ms = 0.f;
+    if (ntried) *ntried = 0;
+    if (m == 0 || n == 0) return 0;
+    reps = std::max(1, std::min(reps, 50));
+    // candidates: the default first (ties keep it), then the sweep axes of
+    // P:L796-824 (tile height; panel-group width for wide matrices)
+    const int64_t leafs[] = {0, 64, 96, 128, 160, 192, 224, 256};
+    std::vector<int64_t> nbs = {0};
+    for (int64_t nb : {32, 64, 96, 128, 160, 192, 224, 256})
+        if (nb < n) nbs.push_back(nb);
+    struct Cand {
+        caqr_opts o;
+        int64_t b, nb;
+        bool chain, skinny;
+        size_t ws;
+    };
+    std::vector<Cand> cands;
+    for (int64_t nb : nbs)
+        for (int64_t lf : leafs) {
+            caqr_opts o{};
+            o.leaf_rows = lf;
+            o.panel_cols = nb;
+            Plan pl;
+            if (make_plan(m, n, dtype, &o, 9, &pl)) continue;
+            bool dup = false;
+            for (const Cand& c : cands)
+                dup |= c.b == pl.b && c.nb == pl.nb && c.chain == pl.chain && c.skinny == pl.skinny;
+            if (!dup) cands.push_back(Cand{o, pl.b, pl.nb, pl.chain, pl.skinny, std::max<size_t>(plan_ws_bytes(pl), 256)});
+        }
+    size_t wsmax = 256;
+    for (const Cand& c : cands) wsmax = std::max(wsmax, c.ws);
+    T *Ac = nullptr, *Rc = nullptr;
+    void* ws = nullptr;
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    cudaError_t e = cudaMalloc(reinterpret_cast<void**>(&Ac), sizeof(T) * (size_t)m * n);
+    if (e == cudaSuccess) e = cudaMalloc(reinterpret_cast<void**>(&Rc), sizeof(T) * (size_t)n * n);
+    if (e == cudaSuccess) e = cudaMalloc(&ws, wsmax);
+    if (e == cudaSuccess) e = cudaEventCreate(&e0);
+    if (e == cudaSuccess) e = cudaEventCreate(&e1);
+    int rc = 0;
+    float bestt = 0.f;
+    int tried = 0;
+    for (size_t ci = 0; ci < cands.size() && e == cudaSuccess && !rc; ++ci) {
+        std::vector<float> ts;
+        for (int r = 0; r <= reps && e == cudaSuccess && !rc; ++r) {  // r = 0: warm-up
+            e = cudaMemcpy2DAsync(Ac, sizeof(T) * m, A, sizeof(T) * lda, sizeof(T) * m, n,
+                                  cudaMemcpyDeviceToDevice, s);
+            if (e == cudaSuccess) e = cudaEventRecord(e0, s);
+            if (e == cudaSuccess)
+                rc = factor_impl<T>(m, n, Ac, m, Rc, n, ws, cands[ci].ws, &cands[ci].o, s, dtype);
+            if (!rc && e == cudaSuccess) e = cudaEventRecord(e1, s);
+            if (!rc && e == cudaSuccess) e = cudaEventSynchronize(e1);
+            float ms = 0.f;
+            if (!rc && e == cudaSuccess) e = cudaEventElapsedTime(&ms, e0, e1);
+            if (r > 0) ts.push_back(ms);
+        }
+        if (rc || e != cudaSuccess) break;
+        std::sort(ts.begin(), ts.end());
+        const float t = ts[ts.size() / 2];
+        ++tried;
+        if (ci == 0 && default_ms) *default_ms = t;
+        if (ci == 0 || t < bestt) {
+            bestt = t;
+            *best = cands[ci].o;
+        }
+    }
+    if (e0) cudaEventDestroy(e0);
+    if (e1) cudaEventDestroy(e1);
+    if (Ac) cudaFree(Ac);
+    if (Rc) cudaFree(Rc);
+    if (ws) cudaFree(ws);
+    if (ntried) *ntried = tried;
+    *best_ms = bestt;
+    if (rc) return rc;
+    if (e != cudaSuccess) {
+        g_last_cuda_error = (int)e;
+        return CAQR_ERR_CUDA;
+    }
+    return 0;
+}
+
 extern "C" {
+
+int caqr_tune(int64_t m, int64_t n, int dtype, const void* A, int64_t lda, int reps, caqr_opts* best,
+              float* best_ms, float* default_ms, int* ntried, caqr_stream_t stream) {
+    if (dtype == CAQR_F32)
+        return tune_impl<float>(m, n, static_cast<const float*>(A), lda, reps, dtype, best, best_ms, default_ms,
+                                ntried, stream);
+    if (dtype == CAQR_F64)
+        return tune_impl<double>(m, n, static_cast<const double*>(A), lda, reps, dtype, best, best_ms, default_ms,
+                                 ntried, stream);
+    return -3;
+}
 
 size_t caqr_workspace_bytes(int64_t m, int64_t n, int dtype, const caqr_opts* opts) {
     if (m < 0 || n < 0 || n > m || (dtype != CAQR_F32 && dtype != CAQR_F64)) return 0;

@@ -65,7 +65,7 @@ def test_plan_info(L):
     assert p["leaves"] == 4465 and p["chains"] == 280 and p["tree_levels"] == 9 and p["panels"] == 6
     assert p["launches"] == 2  # one fused TSQR kernel + extract_r
     p = caqr.caqr_plan_info(8192, 8192)
-    assert p["panel_cols"] == 64 and p["groups"] == 128
+    assert p["panel_cols"] == 128 and p["groups"] == 64 and p["leaf_rows"] == 256  # wide: (b, nb) = (256, 128)
     p = caqr.caqr_plan_info(4096, 16, 0, caqr.make_opts(leaf_rows=128))
     assert p["leaf_rows"] == 128 and p["leaves"] == 32 and p["tree_levels"] == 5
     p = caqr.caqr_plan_info(4_000_000, 8)  # skinny: 256-row tiles, ~2368 chains (16 warps x 148 SMs)

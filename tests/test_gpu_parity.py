@@ -878,3 +878,39 @@ def test_cuda_graph_capture(caqr, m, n):
         g.replay()
         torch.cuda.synchronize()
         assert torch.equal(R, R_e) and torch.equal(C, C_e) and torch.equal(Q, Q_e)
+
+
+@pytest.mark.parametrize("m,n,dtype", [(20_000, 100, np.float32), (4096, 640, np.float32), (30_000, 24, np.float64)])
+def test_tune_plan_search(caqr, m, n, dtype):
+    """caqr_tune: times several distinct plans on
+    a scratch copy, leaves A unchanged, returns a plan no slower than the
+    default (the default is a candidate), and that plan factors A correctly
+    (R^T R = A^T A)."""
+    tdt = torch.float32 if dtype == np.float32 else torch.float64
+    A0 = workloads.device_gaussian(m, n, seed=11, dtype=tdt, device="cuda").t()
+    A = caqr.colmajor_empty(m, n, tdt)
+    A.copy_(A0)
+    opts, best_ms, default_ms, tried = caqr.caqr_tune(A, reps=2)
+    torch.cuda.synchronize()
+    assert torch.equal(A, A0)
+    assert tried >= 3 and 0 < best_ms <= default_ms
+    R, _ = caqr.caqr_factor(A, opts=opts)
+    A64 = A0.double()
+    G = A64.t() @ A64
+    R64 = R.double()
+    err = (R64.t() @ R64 - G).norm() / G.norm()
+    assert err.item() <= BOUNDS[dtype]["res"]  # backward error of a Householder QR (the residual bound)
+    assert torch.tril(R, -1).abs().max().item() == 0.0
+
+
+def test_tune_info_codes(caqr):
+    L = caqr.lib()
+    import ctypes
+
+    best = caqr.Opts()
+    f = ctypes.c_float()
+    assert L.caqr_tune(-1, 4, 0, None, 1, 1, ctypes.byref(best), ctypes.byref(f), None, None, None) == -1
+    assert L.caqr_tune(4, 5, 0, None, 4, 1, ctypes.byref(best), ctypes.byref(f), None, None, None) == -2
+    assert L.caqr_tune(8, 4, 7, None, 8, 1, ctypes.byref(best), ctypes.byref(f), None, None, None) == -3
+    assert L.caqr_tune(8, 4, 0, None, 8, 1, ctypes.byref(best), ctypes.byref(f), None, None, None) == -4
+    assert L.caqr_tune(8, 4, 0, None, 8, 1, None, ctypes.byref(f), None, None, None) == -7
