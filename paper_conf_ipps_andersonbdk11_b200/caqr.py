@@ -51,7 +51,8 @@ def lib() -> ctypes.CDLL:
         if not os.path.exists(LIB_PATH):
             raise RuntimeError(f"{LIB_PATH} missing: run `python -m paper_conf_ipps_andersonbdk11_b200.build` "
                                "(no CPU fallback exists)")
-        L = ctypes.CDLL(LIB_PATH)
+        # CAQR_LIB_PATH: development A/B of alternative builds (tools/ab_time.py)
+        L = ctypes.CDLL(os.environ.get("CAQR_LIB_PATH", LIB_PATH))
         i64, vp, sz, ip = ctypes.c_int64, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int
         op = ctypes.POINTER(Opts)
         L.caqr_workspace_bytes.argtypes = [i64, i64, ip, op]

@@ -33,8 +33,9 @@ if os.environ.get("CAQR_PROFILE") == "1":
     out = (ctypes.c_ulonglong * 16)()
     L.caqr_debug_profile_read.argtypes = [ctypes.c_void_p]
     L.caqr_debug_profile_read(out)
-    names = ["fetch", "wait", "stage_panel", "factor", "store_vform", "G_T", "stage_C", "VtC", "apply", "publish"]
-    tot = sum(out[i] for i in range(10))
-    for i, nm in enumerate(names):
-        print(f"{nm:12s} {out[i] / tot * 100:5.1f}%  {out[i] / 1.965e9 / max(1, a.reps):.4f} CTA-s")
+    names = {0: "fetch", 1: "wait", 2: "stage_panel", 3: "factor", 4: "G=V^T V", 12: "build_t",
+             5: "fence/publish", 6: "stage_C", 7: "VtC", 8: "apply", 9: "publish"}
+    tot = sum(out[i] for i in names)
+    for i, nm in names.items():
+        print(f"{nm:14s} {out[i] / tot * 100:5.1f}%  {out[i] / 1.965e9 / max(1, a.reps):.4f} CTA-s")
     print("leaf panel-steps", out[10], "merge panel-steps", out[11], "total CTA-s", tot / 1.965e9 / a.reps)
