@@ -626,21 +626,35 @@ __device__ __forceinline__ void gemm_vtc(const Grp& G, const T* Vs, const T* Cs,
 template <typename T>
 __device__ __forceinline__ void build_t(const Grp& Gr, const T* G, const T* tau_s, int wp, T* Tt,
                                        T* tglobal = nullptr) {
+    using V4 = typename Vec4<T>::type;
+    constexpr int VN = Vec4<T>::n;
     const int lane = Gr.tid & 31;
     if (Gr.tid >= 32) return;
     T row[32];
 #pragma unroll
     for (int j = 0; j < 32; ++j) {
+        // G is symmetric bit for bit (G[k][j] and G[j][k] are the same products
+        // summed in the same order), so G[k][j] is read from row j: contiguous,
+        // 16-byte broadcast loads (a quarter of the shared-memory instructions
+        // of a column walk, which made this one-warp step LDS-issue bound)
+        const T* gj = G + j * kTS;
         T a0 = 0, a1 = 0, a2 = 0, a3 = 0;
 #pragma unroll
         for (int k = 0; k + 3 < j; k += 4) {
-            a0 = fma(row[k + 0], G[(k + 0) * kTS + j], a0);
-            a1 = fma(row[k + 1], G[(k + 1) * kTS + j], a1);
-            a2 = fma(row[k + 2], G[(k + 2) * kTS + j], a2);
-            a3 = fma(row[k + 3], G[(k + 3) * kTS + j], a3);
+            T g[4];
+#pragma unroll
+            for (int h = 0; h < 4 / VN; ++h) {
+                const V4 q = *reinterpret_cast<const V4*>(gj + k + h * VN);
+#pragma unroll
+                for (int e = 0; e < VN; ++e) g[h * VN + e] = vget<T>(q, e);
+            }
+            a0 = fma(row[k + 0], g[0], a0);
+            a1 = fma(row[k + 1], g[1], a1);
+            a2 = fma(row[k + 2], g[2], a2);
+            a3 = fma(row[k + 3], g[3], a3);
         }
 #pragma unroll
-        for (int k = j & ~3; k < j; ++k) a0 = fma(row[k], G[k * kTS + j], a0);
+        for (int k = j & ~3; k < j; ++k) a0 = fma(row[k], gj[k], a0);
         const T tau = j < wp ? tau_s[j] : T(0);
         row[j] = (j == lane) ? tau : (j > lane ? -tau * ((a0 + a1) + (a2 + a3)) : T(0));
     }
