@@ -571,6 +571,201 @@ __device__ __forceinline__ void factor_panel_wb4(const Grp& G, T* P, int RGP, in
 }
 
 // ---------------------------------------------------------------------------
+// Panel factorization, reflector-pipelined ("PIPE").  Same ownership as WB4
+// (warp w owns panel columns 4(7-w) .. +3, lane l rows l + 32 i), but no CTA
+// barrier per block: reflector j is published (v_j in P[:, j], tau_j) through
+// its own shared-memory mbarrier, and every warp that owns later columns
+// applies H_j = I - tau_j v_j v_j^T to them as soon as it arrives (the
+// unblocked xGEQR2 order).  The next block's owner has applied
+// all but the newest reflector when its turn comes, so the hand-off costs one
+// reflector application instead of a barrier plus a 4-reflector block update.
+// The owner's own block: one warp reduction per reflector gives the squared
+// norm and the dots with the block's later columns (WB4's unscaled-column
+// trick); the compact-WY T comes afterwards from G = V^T V (build_t).
+// mb: 32 mbarriers (arrival count 1), `parity` = this call's phase (each call
+// arrives exactly once on every one of them, including columns >= wp).
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void mbar_arrive1(uint64_t* mb) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"((unsigned)__cvta_generic_to_shared(mb))
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_wait_parity(uint64_t* mb, unsigned parity) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "PIPE_WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra PIPE_WAIT_%=;\n}" ::"r"((unsigned)__cvta_generic_to_shared(mb)),
+        "r"(parity)
+        : "memory");
+}
+// All-lane sum of N values by a SHFL butterfly (N <= 4: fewer dependent steps
+// than the shared-memory transpose of warp_reduce_many).
+template <int N, typename T>
+__device__ __forceinline__ void warp_allsum_bfly(T (&v)[N]) {
+#pragma unroll
+    for (int o = 16; o >= 1; o >>= 1)
+#pragma unroll
+        for (int k = 0; k < N; ++k) v[k] += __shfl_xor_sync(0xffffffffu, v[k], o);
+}
+
+template <typename T>
+__device__ __forceinline__ void factor_panel_pipe(const Grp& G, T* P, int RGP, int RG, int wp, T* tau_s,
+                                                  uint64_t* mb, unsigned parity, const NodeRows* out_nr,
+                                                  T* out_A, int64_t out_lda, int64_t out_c0, int out_p) {
+    const int warp = G.tid >> 5, lane = G.tid & 31;
+    const int blk = __shfl_sync(0xffffffffu, kWarps - 1 - warp, 0);
+    const int cb = 4 * blk;
+    const int nc = max(0, min(4, wp - cb));
+    // every warp reads and (as owner) writes only its own columns of P: no
+    // barrier needed before the loads
+    T x[4][8];
+#pragma unroll
+    for (int q = 0; q < 4; ++q)
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            const int r = lane + 32 * i;
+            x[q][i] = (q < nc && r < RG) ? P[(size_t)(cb + q) * RGP + padr<T>(r)] : T(0);
+        }
+    if (nc > 0) {
+        // ---- earlier reflectors, one at a time as they are published ----
+        for (int jr = 0; jr < cb; ++jr) {
+            mbar_wait_parity(&mb[jr], parity);
+            const T tau = tau_s[jr];
+            if (tau == T(0)) continue;
+            T v[8];
+#pragma unroll
+            for (int i = 0; i < 8; ++i) v[i] = P[(size_t)jr * RGP + padr<T>(lane + 32 * i)];
+            T d[4];
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                T a0 = T(0), a1 = T(0);
+#pragma unroll
+                for (int i = 0; i < 8; i += 2) {
+                    a0 = fma(v[i], x[q][i], a0);
+                    a1 = fma(v[i + 1], x[q][i + 1], a1);
+                }
+                d[q] = a0 + a1;
+            }
+            warp_allsum_bfly<4>(d);
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const T st = tau * d[q];
+#pragma unroll
+                for (int i = 0; i < 8; ++i) x[q][i] = fma(-st, v[i], x[q][i]);
+            }
+        }
+        // ---- this warp's block: reflectors cb .. cb + nc - 1 ----
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            if (q < nc) {
+                const int j = cb + q;
+                // slot 0: ||x_q (rows > j)||^2, slot 1 + m: x_q . x_{q+1+m} (rows > j)
+                T red[4] = {T(0), T(0), T(0), T(0)};
+#pragma unroll
+                for (int i = 0; i < 8; ++i) {
+                    const int r = lane + 32 * i;
+                    const T xq = r > j ? x[q][i] : T(0);
+                    red[0] = fma(xq, xq, red[0]);
+#pragma unroll
+                    for (int m = 0; m < 3; ++m)
+                        if (m < 3 - q) red[1 + m] = fma(xq, x[q + 1 + m][i], red[1 + m]);
+                }
+                if (q == 0) warp_allsum_bfly<4>(red);
+                else if (q == 1) {
+                    T rr[3] = {red[0], red[1], red[2]};
+                    warp_allsum_bfly<3>(rr);
+                    red[0] = rr[0]; red[1] = rr[1]; red[2] = rr[2];
+                } else if (q == 2) {
+                    T rr[2] = {red[0], red[1]};
+                    warp_allsum_bfly<2>(rr);
+                    red[0] = rr[0]; red[1] = rr[1];
+                } else {
+                    T rr[1] = {red[0]};
+                    warp_allsum_bfly<1>(rr);
+                    red[0] = rr[0];
+                }
+                const T al = __shfl_sync(0xffffffffu, x[q][0], j);
+                T head[3];
+#pragma unroll
+                for (int m = 0; m < 3; ++m)
+                    head[m] = (m < 3 - q) ? __shfl_sync(0xffffffffu, x[q + 1 + m][0], j) : T(0);
+                const T sg = red[0];
+                T tau = T(0), beta = al, scale = T(1);
+                if (j < RG && sg != T(0)) {
+                    const T ss = fma(al, al, sg);
+                    const T aa = fabs(al);
+                    T rmu, mu;
+                    rsqrt_refined(ss, rmu, mu);
+                    beta = -copysign(mu, al);
+                    tau = fma(aa, rmu, T(1));
+                    scale = copysign(rcp_refined(aa + mu), al);
+                }
+                T v[8];
+#pragma unroll
+                for (int i = 0; i < 8; ++i) {
+                    const int r = lane + 32 * i;
+                    if (r > j) x[q][i] *= scale;
+                    if (r == j) x[q][i] = beta;
+                    v[i] = r > j ? x[q][i] : (r == j ? T(1) : T(0));
+                    P[(size_t)j * RGP + padr<T>(r)] = v[i];
+                }
+                if (lane == 0) tau_s[j] = tau;
+                __syncwarp();
+                if (lane == 0) mbar_arrive1(&mb[j]);  // release: v_j and tau_j are visible
+#pragma unroll
+                for (int m = 0; m < 3; ++m) {
+                    if (m < 3 - q && tau != T(0)) {  // H_j on the block's later column q + 1 + m
+                        const T st = tau * fma(scale, red[1 + m], head[m]);
+#pragma unroll
+                        for (int i = 0; i < 8; ++i) x[q + 1 + m][i] = fma(-st, v[i], x[q + 1 + m][i]);
+                    }
+                }
+            }
+        }
+    }
+    // reflectors this call does not produce (columns >= wp) still complete
+    // their phase, so every mbarrier advances exactly once per call
+    if (lane == 0)
+        for (int q = nc; q < 4; ++q) mbar_arrive1(&mb[cb + q]);
+    gsync(G);  // every reflector applied: P's v columns are no longer read
+    {
+        // epilogue straight from registers (as factor_panel_wb4): the stored
+        // form (R / v, structure masks) to global, the V form into P
+        const NodeRows& nr = *out_nr;
+        int64_t grow[8];
+        int key[8];
+        bool seg0[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            const int r = lane + 32 * i;
+            seg0[i] = r < nr.n0;
+            grow[i] = seg0[i] ? nr.r0 + r : nr.r1 + (r - nr.n0);
+            key[i] = seg0[i] ? (nr.seg0_tri ? r : -1) : (nr.seg1_upper ? r - nr.n0 - 32 * out_p : -1);
+        }
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            const int jj = cb + q;
+            T* col = out_A + (out_c0 + jj) * out_lda;
+            T* pcol = P + (size_t)jj * RGP;
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                const int r = lane + 32 * i;
+                const bool in = q < nc && r < RG;
+                const bool stored = key[i] <= jj;
+                if (in && stored) col[grow[i]] = x[q][i];
+                T v = T(0);
+                if (in) {
+                    if (seg0[i]) v = nr.seg0_tri ? (r == jj ? T(1) : T(0)) : (r > jj ? x[q][i] : (r == jj ? T(1) : T(0)));
+                    else v = stored ? x[q][i] : T(0);
+                }
+                pcol[padr<T>(r)] = v;
+            }
+        }
+    }
+    gsync(G);
+}
+
+// ---------------------------------------------------------------------------
 // W(32 x 32) = V^T C over RG rows, V and C padded-column tiles (32 columns).
 // 8 warps = 4-way split of the rows x 2 column halves; deterministic reduction.
 // ---------------------------------------------------------------------------
@@ -1115,6 +1310,14 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
     const bool vec = sizeof(T) == 4 && (reinterpret_cast<uintptr_t>(A) % 16 == 0) && (g.lda % 4 == 0) &&
                      (g.row0 % 4 == 0) && (g.b % 4 == 0) && (g.bm % 4 == 0);
     __shared__ int s_task;
+#ifndef CAQR_PANEL_WB4
+    __shared__ __align__(8) uint64_t s_mb[32];  // per-reflector publication (factor_panel_pipe)
+    unsigned pipe_parity = 0;
+    if (threadIdx.x < 32)
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"((unsigned)__cvta_generic_to_shared(&s_mb[threadIdx.x]))
+                     : "memory");
+    __syncthreads();
+#endif
     const Grp G0{(int)threadIdx.x, 0};
     int* ticket = sync;
     int* flags = sync + 32;  // [L][npan]
@@ -1142,6 +1345,12 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
         if (threadIdx.x == 0) s_task = atomicAdd(ticket, 1);
         __syncthreads();
         const int64_t task = s_task;
+        if (prof && threadIdx.x == 0) {  // timeline: first start, last chain end, last merge end
+            unsigned long long gt;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt));
+            if (task == 0) atomicMax(prof + 15, ~gt);
+            atomicMax(prof + 14, gt);
+        }
         if (task >= total) break;
         int level = -1;
         int64_t node = task;
@@ -1251,7 +1460,12 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
             if (threadIdx.x < 32) tau_s[threadIdx.x] = T(0);
             __syncthreads();
             CAQR_PROF(2);
+#ifdef CAQR_PANEL_WB4
             factor_panel_wb4<T>(G0, P, RGP, RG, wp, tau_s, Wp, Cs, &nr, A, g.lda, c0, p);
+#else
+            factor_panel_pipe<T>(G0, P, RGP, RG, wp, tau_s, s_mb, pipe_parity, &nr, A, g.lda, c0, p);
+            pipe_parity ^= 1u;
+#endif
             CAQR_PROF(3);
             gemm_vtc(G0, P, P, RGP, R32, Wp, W);  // G = V^T V
             CAQR_PROF(4);
@@ -1309,6 +1523,11 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
             if (threadIdx.x == 0 && kt == ntile - 1)  // panel p's trailing update done
                 st_release(flags + slot_a * g.npan + p, 2 * (level < 0 ? 1 : my_ver));
             CAQR_PROF(9);
+        }
+        if (prof && threadIdx.x == 0 && level < 0) {  // timeline: this chain's end
+            unsigned long long gt;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt));
+            atomicMax(prof + 13, gt);
         }
     }
     if (prof && threadIdx.x == 0)

@@ -39,3 +39,6 @@ if os.environ.get("CAQR_PROFILE") == "1":
     for i, nm in names.items():
         print(f"{nm:14s} {out[i] / tot * 100:5.1f}%  {out[i] / 1.965e9 / max(1, a.reps):.4f} CTA-s")
     print("leaf panel-steps", out[10], "merge panel-steps", out[11], "total CTA-s", tot / 1.965e9 / a.reps)
+    t0 = (2**64 - 1) - out[15]
+    print(f"timeline (last rep): chains done by {(out[13] - t0) / 1e3:.1f} us (last chain end), "
+          f"kernel end {(out[14] - t0) / 1e3:.1f} us")
