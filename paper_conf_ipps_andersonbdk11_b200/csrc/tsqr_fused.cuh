@@ -646,7 +646,7 @@ __device__ __forceinline__ void factor_panel_pipe(const Grp& G, T* P, int RGP, i
                 }
                 d[q] = a0 + a1;
             }
-            warp_allsum_bfly<4>(d);
+            warp_allsum_bfly<4>(d);  // (a shared-memory transpose instead: 5.55 vs 5.37 ms)
 #pragma unroll
             for (int q = 0; q < 4; ++q) {
                 const T st = tau * d[q];

@@ -135,7 +135,7 @@ __device__ __forceinline__ void factor_panel_timed(T* P, int RGP, int RG, int wp
 
 template <typename T>
 __device__ __forceinline__ void factor_panel_wb4_timed(T* P, int RGP, int RG, int wp, T* tau_s, T* Tb, unsigned long long* tm) {
-    T* scr_all = P + 32 * 324 + 1024;
+    T* scr_all = P + 32 * RGP + 1024;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     // block blk = 7 - warp: the warp that owns the next block always has the
     // highest warp id among the warps still applying the current one, so the
@@ -341,6 +341,10 @@ __global__ void __launch_bounds__(256, 2) bench(float* data, int RG, int reps, u
     float* tau_s = P + 32 * RGP;
     unsigned long long total = 0;
     __shared__ unsigned long long tm[8];
+    __shared__ __align__(8) uint64_t mbs[32];
+    if (threadIdx.x < 32)
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"((unsigned)__cvta_generic_to_shared(&mbs[threadIdx.x])) : "memory");
+    unsigned par = 0;
     if (threadIdx.x < 8) tm[threadIdx.x] = 0;
     __syncthreads();
     for (int r = 0; r < reps; ++r) {
@@ -352,7 +356,12 @@ __global__ void __launch_bounds__(256, 2) bench(float* data, int RG, int reps, u
         __syncthreads();
         const unsigned long long t0 = clock64();
         if (MODE == 1) factor_panel_timed<float, 8>(P, RGP, RG, 32, tau_s, tm);
-        else if (MODE == 2) factor_panel_wb4<float>(Grp{(int)threadIdx.x, 0}, P, RGP, RG, 32, tau_s, tau_s + 32, P + 32 * 324 + 1024);
+        else if (MODE == 2) factor_panel_wb4<float>(Grp{(int)threadIdx.x, 0}, P, RGP, RG, 32, tau_s, tau_s + 32, P + 32 * RGP + 1024);
+        else if (MODE == 6) {
+            NodeRows nr{0, 0, 256, 0, 0, 0, 0};
+            factor_panel_pipe<float>(Grp{(int)threadIdx.x, 0}, P, RGP, RG, 32, tau_s, mbs, par, &nr, data + 4 * 8192, 256, 0, 0);
+            par ^= 1u;
+        }
         else if (MODE == 3) factor_panel_wb4_timed<float>(P, RGP, RG, 32, tau_s, tau_s + 32, tm);
         else factor_panel_regs<float, 8>(P, RGP, RG, 32, tau_s);
         const unsigned long long t1 = clock64();
@@ -367,7 +376,7 @@ __global__ void __launch_bounds__(256, 2) bench(float* data, int RG, int reps, u
 int main() {
     float* d;
     unsigned long long* cyc;
-    cudaMalloc(&d, 4 * 8192 * sizeof(float));
+    cudaMalloc(&d, 4 * 8192 * sizeof(float) + 256 * 32 * sizeof(float));
     cudaMalloc(&cyc, 4096 * sizeof(unsigned long long));
     float h[4 * 8192];
     unsigned s = 1;
@@ -401,6 +410,18 @@ int main() {
         for (int i = 0; i < grid; ++i) avg += hc2[i];
         avg /= grid;
         printf("WB4 grid %4d: %8.0f cycles/panel = %6.0f cycles/column (%s)\n", grid, avg, avg / 32,
+               cudaGetErrorString(cudaGetLastError()));
+    }
+    cudaFuncSetAttribute(bench<6>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    for (int grid : {1, 148, 296}) {
+        bench<6><<<grid, 256, smem>>>(d, 256, 20, cyc);
+        cudaDeviceSynchronize();
+        unsigned long long hc6[512];
+        cudaMemcpy(hc6, cyc, grid * sizeof(unsigned long long), cudaMemcpyDeviceToHost);
+        double avg = 0;
+        for (int i = 0; i < grid; ++i) avg += hc6[i];
+        avg /= grid;
+        printf("PIPE grid %4d: %8.0f cycles/panel = %6.0f cycles/column (%s)\n", grid, avg, avg / 32,
                cudaGetErrorString(cudaGetLastError()));
     }
     cudaFuncSetAttribute(bench<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
