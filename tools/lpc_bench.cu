@@ -7,7 +7,7 @@
 #include <cuda_runtime.h>
 
 #include "panel_lpc.cuh"
-#include "../paper_conf_ipps_andersonbdk11_b200/csrc/tsqr_fused.cuh"
+#include "panel_variants.cuh"
 
 using namespace caqr;
 

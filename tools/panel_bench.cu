@@ -4,7 +4,7 @@
 #include <cstdio>
 #include <cuda_runtime.h>
 
-#include "../paper_conf_ipps_andersonbdk11_b200/csrc/tsqr_fused.cuh"
+#include "panel_variants.cuh"
 
 using namespace caqr;
 
