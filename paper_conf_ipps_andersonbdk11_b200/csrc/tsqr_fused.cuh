@@ -137,6 +137,26 @@ __device__ __forceinline__ void gsync(const Grp& g) {
 // stores its N partials, lane l sums value l % NP over a group of NP rows, a
 // few shuffles combine the groups, and the totals are broadcast back.
 // `scr` is this warp's private scratch of 32 * (NP + 4) + NP elements.
+// As warp_reduce_many, but each lane only needs one total: lane l returns the
+// sum of value l % NP (no broadcast back through shared memory).
+template <int N, typename T>
+__device__ __forceinline__ T warp_reduce_scatter_smem(const T (&v)[N], T* scr) {
+    constexpr int NP = N <= 1 ? 1 : N <= 2 ? 2 : N <= 4 ? 4 : N <= 8 ? 8 : N <= 16 ? 16 : 32;
+    constexpr int LD = NP + 4;
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int k = 0; k < NP; ++k) scr[lane * LD + k] = k < N ? v[k] : T(0);
+    __syncwarp();
+    const int k = lane % NP, g = lane / NP;
+    T acc = T(0);
+#pragma unroll
+    for (int r = 0; r < NP; ++r) acc += scr[(g * NP + r) * LD + k];
+#pragma unroll
+    for (int o = NP; o < 32; o <<= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    __syncwarp();
+    return acc;
+}
+
 template <int N, typename T>
 __device__ __forceinline__ void warp_reduce_many(T (&v)[N], T* scr) {
     constexpr int NP = N <= 1 ? 1 : N <= 2 ? 2 : N <= 4 ? 4 : N <= 8 ? 8 : N <= 16 ? 16 : 32;
@@ -201,7 +221,8 @@ __device__ __forceinline__ void warp_allsum_bfly(T (&v)[N]) {
 template <typename T>
 __device__ __forceinline__ void factor_panel_pipe(const Grp& G, T* P, int RGP, int RG, int wp, T* tau_s,
                                                   uint64_t* mb, unsigned parity, const NodeRows* out_nr,
-                                                  T* out_A, int64_t out_lda, int64_t out_c0, int out_p) {
+                                                  T* out_A, int64_t out_lda, int64_t out_c0, int out_p,
+                                                  T* Gout = nullptr, T* scr_all = nullptr) {
     const int warp = G.tid >> 5, lane = G.tid & 31;
     const int blk = __shfl_sync(0xffffffffu, kWarps - 1 - warp, 0);
     const int cb = 4 * blk;
@@ -317,6 +338,64 @@ __device__ __forceinline__ void factor_panel_pipe(const Grp& G, T* P, int RGP, i
     // their phase, so every mbarrier advances exactly once per call
     if (lane == 0)
         for (int q = nc; q < 4; ++q) mbar_arrive1(&mb[cb + q]);
+    if (Gout && nc > 0) {
+        // The Gram matrix G = V^T V for the compact-WY T (build_t reads G[j][k],
+        // k < j), by warps whose own columns are final while the later blocks are
+        // still being factored: this block's 6 entries, then, as each later block
+        // completes (its last mbarrier), the 4 x 4 entries against it.  Exact
+        // fp32 dots over the panel rows, as the separate G = V^T V pass was.
+        T v[4][8];
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                const int r = lane + 32 * i, j = cb + q;
+                v[q][i] = q < nc ? (r > j ? x[q][i] : (r == j ? T(1) : T(0))) : T(0);
+            }
+        T* scr = scr_all + warp * (32 * 20 + 16);
+        {
+            T gw[6];
+            int e = 0;
+#pragma unroll
+            for (int a = 0; a < 4; ++a)
+#pragma unroll
+                for (int b = a + 1; b < 4; ++b, ++e) {
+                    T acc = T(0);
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) acc = fma(v[a][i], v[b][i], acc);
+                    gw[e] = acc;
+                }
+            const T gl = warp_reduce_scatter_smem<6>(gw, scr);  // lane l: entry l % 8
+            if (lane < 6) {
+                const int a = lane < 3 ? 0 : (lane < 5 ? 1 : 2);
+                const int b = lane < 3 ? lane + 1 : (lane < 5 ? lane - 1 : 3);
+                Gout[(cb + b) * kTS + cb + a] = gl;
+            }
+        }
+        const int nblk = (wp + 3) / 4;
+        for (int bb = blk + 1; bb < nblk; ++bb) {
+            mbar_wait_parity(&mb[4 * bb + 3], parity);  // block bb complete
+            T w[16];
+#pragma unroll
+            for (int qb = 0; qb < 4; ++qb) {
+                T vb[8];
+#pragma unroll
+                for (int i = 0; i < 8; ++i) vb[i] = P[(size_t)(4 * bb + qb) * RGP + padr<T>(lane + 32 * i)];
+#pragma unroll
+                for (int qa = 0; qa < 4; ++qa) {
+                    T acc = T(0);
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) acc = fma(v[qa][i], vb[i], acc);
+                    w[qa * 4 + qb] = acc;
+                }
+            }
+            const T wl = warp_reduce_scatter_smem<16>(w, scr);  // lane l: entry l % 16
+            if (lane < 16) Gout[(4 * bb + (lane & 3)) * kTS + cb + (lane >> 2)] = wl;
+        }
+    }
+    if (Gout && nc == 0)  // blocks beyond wp: zero rows (build_t multiplies them by tau = 0)
+#pragma unroll
+        for (int q = 0; q < 4; ++q) Gout[(cb + q) * kTS + lane] = T(0);
     gsync(G);  // every reflector applied: P's v columns are no longer read
     {
         // epilogue straight from registers (as factor_panel_wb4): the stored
@@ -1048,10 +1127,16 @@ tsqr_fused_kernel(Geom g, T* A, T* __restrict__ Tws, int* __restrict__ sync, int
             if (threadIdx.x < 32) tau_s[threadIdx.x] = T(0);
             __syncthreads();
             CAQR_PROF(2);
+#ifdef CAQR_NO_PIPE_GRAM
             factor_panel_pipe<T>(G0, P, RGP, RG, wp, tau_s, s_mb, pipe_parity, &nr, A, g.lda, c0, p);
+#else
+            factor_panel_pipe<T>(G0, P, RGP, RG, wp, tau_s, s_mb, pipe_parity, &nr, A, g.lda, c0, p, W, Cs);
+#endif
             pipe_parity ^= 1u;
             CAQR_PROF(3);
+#ifdef CAQR_NO_PIPE_GRAM
             gemm_vtc(G0, P, P, RGP, R32, Wp, W);  // G = V^T V
+#endif
             CAQR_PROF(4);
             build_t(G0, W, tau_s, wp, Tt, Tws + nr.tblk * (kPW * kPW));
             __syncthreads();
