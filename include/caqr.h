@@ -267,6 +267,50 @@ int caqr_dist_combine_blocks_f64(int P, int64_t n, const double *blocks, double 
  * accepts caqr_dist_destroy.  -1: h NULL; CAQR_ERR_CUDA: the stream failed. */
 int caqr_dist_wait(caqr_dist *h, caqr_stream_t stream, int timeout_ms);
 
+/* Peer-memory exchange of the local R factors -- the alternative to the NCCL
+ * all-gather of caqr_dist_factor, with the exchange fused into the restack of
+ * the combine's input (distributed TSQR; the paper's one-kernel-
+ * per-step dataflow, carried across GPUs).  Rank `rank` of P:
+ *   1. stores its n x n R (R, ldr; column-major) into slot `rank` of buffer
+ *      (epoch & 1) of every rank q's mailbox (peer_mailbox[q], NVLink peer
+ *      stores for q != rank);
+ *   2. publishes peer_flags[q][rank] = epoch (system fence, then a
+ *      system-scope release store);
+ *   3. waits (acquire) for its own flags[q] >= epoch from every q and moves
+ *      rank q's block to rows [q n, (q+1) n) of `gather` ((P n) x n,
+ *      ld = P n, column-major), which caqr_combine_* then factors in place.
+ * All P ranks must call it with the same P, n and epoch (1, 2, 3, ... one per
+ * exchange; flags zeroed once before the first).  peer_mailbox / peer_flags:
+ * DEVICE arrays of P device pointers (rank q's mailbox of
+ * caqr_peer_mailbox_bytes(P, n, dtype) bytes and its P ints), mapped into this
+ * process (caqr_ipc_open); the two mailbox buffers let a rank run ahead by
+ * one exchange.  One CTA per peer, asynchronous on `stream`.
+ * status (device int, may be NULL): set to CAQR_ERR_TIMEOUT if a wait exceeded
+ * timeout_ms (> 0; 0 = wait forever) -- `gather` is then invalid.
+ * info: -1 P < 1, -2 rank, -3 n (0..256), -4 R, -5 ldr, -6 peer_mailbox,
+ * -7 peer_flags, -8 gather, -9 epoch < 1; CAQR_ERR_CUDA. */
+size_t caqr_peer_mailbox_bytes(int P, int64_t n, int dtype);
+int caqr_peer_exchange_f32(int P, int rank, int64_t n, const float *R, int64_t ldr, float *const *peer_mailbox,
+                           int *const *peer_flags, float *gather, int epoch, int *status, int timeout_ms,
+                           caqr_stream_t stream);
+int caqr_peer_exchange_f64(int P, int rank, int64_t n, const double *R, int64_t ldr, double *const *peer_mailbox,
+                           int *const *peer_flags, double *gather, int epoch, int *status, int timeout_ms,
+                           caqr_stream_t stream);
+/* The same exchange for P virtual ranks on ONE device (tests; a single
+ * cooperative launch of P x P CTAs, CTA (q, r) playing rank r's sender to /
+ * receiver from q, since ranks that wait on one another must be co-resident):
+ * Rs / mailboxes / flags / gathers: device arrays of P device pointers. */
+int caqr_peer_exchange_emulate_f32(int P, int64_t n, const float *const *Rs, int64_t ldr, float *const *mailboxes,
+                                   int *const *flags, float *const *gathers, int epoch, caqr_stream_t stream);
+int caqr_peer_exchange_emulate_f64(int P, int64_t n, const double *const *Rs, int64_t ldr,
+                                   double *const *mailboxes, int *const *flags, double *const *gathers, int epoch,
+                                   caqr_stream_t stream);
+/* CUDA IPC of a device allocation (peer pointers across processes): the handle
+ * is 64 opaque bytes.  0 / -1 / -2 / CAQR_ERR_CUDA. */
+int caqr_ipc_handle(const void *dptr, void *out64);
+int caqr_ipc_open(const void *handle64, void **dptr);
+int caqr_ipc_close(void *dptr);
+
 /* ---- Least squares through the factorization -------------
  * min ||A x - b||_2 for tall full-rank A, the use of QR the paper opens with
  * (P:L86-92), with LAPACK xGELS semantics: B <- Q^T B, then rows 0..n-1 of B

@@ -115,6 +115,20 @@ def lib() -> ctypes.CDLL:
             f = getattr(L, f"caqr_dist_combine_blocks_{suf}")
             f.argtypes = [ip, i64, vp, vp, i64, vp, i64, vp, sz, vp]
             f.restype = ip
+            f = getattr(L, f"caqr_peer_exchange_{suf}")
+            f.argtypes = [ip, ip, i64, vp, i64, vp, vp, vp, ip, vp, ip, vp]
+            f.restype = ip
+            f = getattr(L, f"caqr_peer_exchange_emulate_{suf}")
+            f.argtypes = [ip, i64, vp, i64, vp, vp, vp, ip, vp]
+            f.restype = ip
+        L.caqr_peer_mailbox_bytes.argtypes = [ip, i64, ip]
+        L.caqr_peer_mailbox_bytes.restype = sz
+        L.caqr_ipc_handle.argtypes = [vp, vp]
+        L.caqr_ipc_handle.restype = ip
+        L.caqr_ipc_open.argtypes = [vp, ctypes.POINTER(vp)]
+        L.caqr_ipc_open.restype = ip
+        L.caqr_ipc_close.argtypes = [vp]
+        L.caqr_ipc_close.restype = ip
         fl = ctypes.c_float
         for suf in ("f32", "f64"):
             f = getattr(L, f"caqr_lstsq_{suf}")
@@ -420,6 +434,70 @@ def caqr_dist_combine_blocks(blocks, P: int, n: int, gather=None, R=None, cws=No
                                                                cws.data_ptr(), cws.numel(), _stream(stream))
     _check(f"caqr_dist_combine_blocks_{suf}", info)
     return R, gather, cws
+
+
+def caqr_peer_mailbox_bytes(P: int, n: int, dtype_code: int) -> int:
+    return int(lib().caqr_peer_mailbox_bytes(P, n, dtype_code))
+
+
+def _ptr_array(ptrs, device):
+    """Device array of raw device pointers (int64), for the pointer-array arguments."""
+    torch = _torch()
+    return torch.tensor([int(p) for p in ptrs], dtype=torch.int64, device=device)
+
+
+def caqr_peer_exchange(P: int, rank: int, R, peer_mailbox, peer_flags, gather, epoch: int, status=None,
+                       timeout_ms: int = 0, stream=None):
+    """caqr_peer_exchange_*: this rank's R into every rank's mailbox (peer
+    stores), flags, and the P blocks restacked into `gather` ((P n) x n).
+    peer_mailbox / peer_flags: int64 device tensors of P device pointers."""
+    code, suf = _dtype_code(R)
+    n = R.shape[1]
+    pr, ldr = _colmajor(R, "R")
+    pg, _ = _colmajor(gather, "gather")
+    info = getattr(lib(), f"caqr_peer_exchange_{suf}")(P, rank, n, pr, ldr, peer_mailbox.data_ptr(),
+                                                        peer_flags.data_ptr(), pg, int(epoch),
+                                                        status.data_ptr() if status is not None else None,
+                                                        int(timeout_ms), _stream(stream))
+    _check(f"caqr_peer_exchange_{suf}", info)
+    return gather
+
+
+def caqr_peer_exchange_emulate(Rs, mailboxes, flags, gathers, epoch: int, stream=None):
+    """The exchange among len(Rs) virtual ranks on one device (tests): Rs,
+    mailboxes, flags, gathers are per-rank tensors (same n, same ldr)."""
+    P = len(Rs)
+    code, suf = _dtype_code(Rs[0])
+    n = Rs[0].shape[1]
+    ldr = _colmajor(Rs[0], "R")[1]
+    for r in Rs:
+        if _colmajor(r, "R")[1] != ldr:
+            raise ValueError("Rs: one leading dimension")
+    dev = Rs[0].device
+    arrs = [_ptr_array([t.data_ptr() for t in ts], dev) for ts in (Rs, mailboxes, flags, gathers)]
+    info = getattr(lib(), f"caqr_peer_exchange_emulate_{suf}")(P, n, arrs[0].data_ptr(), ldr, arrs[1].data_ptr(),
+                                                                arrs[2].data_ptr(), arrs[3].data_ptr(), int(epoch),
+                                                                _stream(stream))
+    _check(f"caqr_peer_exchange_emulate_{suf}", info)
+    # the pointer arrays are temporaries: keep them alive until the launch ran
+    (stream if stream is not None else _torch().cuda.current_stream(dev)).synchronize()
+    return gathers
+
+
+def caqr_ipc_handle(t) -> bytes:
+    buf = ctypes.create_string_buffer(64)
+    _check("caqr_ipc_handle", lib().caqr_ipc_handle(t.data_ptr(), buf))
+    return buf.raw
+
+
+def caqr_ipc_open(handle: bytes) -> int:
+    p = ctypes.c_void_p()
+    _check("caqr_ipc_open", lib().caqr_ipc_open(handle, ctypes.byref(p)))
+    return int(p.value)
+
+
+def caqr_ipc_close(ptr: int):
+    _check("caqr_ipc_close", lib().caqr_ipc_close(ctypes.c_void_p(ptr)))
 
 
 # ---- application layer: SVD via QR, robust PCA (include/caqr.h, Sec. VI) ----

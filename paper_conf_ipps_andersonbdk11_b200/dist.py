@@ -170,3 +170,90 @@ class DistTSQR:
             self.close()
         except Exception:
             pass
+
+
+class PeerTSQR:
+    """Row-sharded TSQR whose R exchange is ``caqr_peer_exchange_*`` -- each rank
+    stores its n x n R straight into every rank's mailbox over NVLink (CUDA IPC
+    peer pointers) and raises a flag; the receive side restacks the P blocks into
+    the combine's input in the same kernel -- instead of the NCCL all-gather of
+    DistTSQR.  Same result bits as DistTSQR (same local factor, same combine).
+
+    Construction maps every rank's mailbox (caqr_peer_mailbox_bytes) and flag
+    array into every process (caqr_ipc_handle / caqr_ipc_open, handles swapped
+    with torch.distributed.all_gather_object), so it needs one process per GPU on
+    one node with peer access.  n and the dtype are fixed per instance."""
+
+    def __init__(self, n: int, dtype=None, group=None, timeout_ms: int = 60000):
+        import torch
+        import torch.distributed as dist
+
+        from . import caqr
+
+        self.caqr = caqr
+        self.group = group
+        self.n = n
+        self.dtype = dtype or torch.float32
+        self.world = dist.get_world_size(group)
+        self.rank = dist.get_rank(group)
+        self.timeout_ms = timeout_ms
+        dev = torch.device("cuda", torch.cuda.current_device())
+        code, _ = caqr._dtype_code(torch.empty(0, dtype=self.dtype))
+        self.code = code
+        self.mailbox = torch.empty(max(caqr.caqr_peer_mailbox_bytes(self.world, n, code), 16), dtype=torch.uint8,
+                                   device=dev)
+        self.flags = torch.zeros(max(self.world, 4), dtype=torch.int32, device=dev)
+        self.status = torch.zeros(1, dtype=torch.int32, device=dev)
+        torch.cuda.synchronize()
+        mine = (caqr.caqr_ipc_handle(self.mailbox), caqr.caqr_ipc_handle(self.flags))
+        allh = [None] * self.world
+        dist.all_gather_object(allh, mine, group=group)
+        self.opened = []
+        mb, fl = [], []
+        for q, (hm, hf) in enumerate(allh):
+            if q == self.rank:
+                mb.append(self.mailbox.data_ptr())
+                fl.append(self.flags.data_ptr())
+            else:
+                pm, pf = caqr.caqr_ipc_open(hm), caqr.caqr_ipc_open(hf)
+                self.opened += [pm, pf]
+                mb.append(pm)
+                fl.append(pf)
+        self.mb_ptrs = caqr._ptr_array(mb, dev)
+        self.fl_ptrs = caqr._ptr_array(fl, dev)
+        self.epoch = 0
+        dist.barrier(group=group)  # every rank's flags are zero before the first exchange
+
+    def factor(self, A_local, opts=None, stream=None):
+        """Factor the local column-major shard in place; returns (R, ws, gather,
+        cws) exactly as DistTSQR.factor.  Raises CaqrError (CAQR_ERR_TIMEOUT)
+        if some rank's block did not arrive within timeout_ms."""
+        import torch
+
+        c = self.caqr
+        m, n = A_local.shape
+        if n != self.n or A_local.dtype != self.dtype:
+            raise ValueError(f"PeerTSQR built for n = {self.n}, {self.dtype}")
+        agree_shards(m, n, self.group)
+        Rl, ws = c.caqr_factor(A_local, opts=opts, stream=stream)
+        self.epoch += 1
+        gather = c.colmajor_empty(self.world * n, n, A_local.dtype, A_local.device)
+        c.caqr_peer_exchange(self.world, self.rank, Rl, self.mb_ptrs, self.fl_ptrs, gather, self.epoch,
+                             status=self.status, timeout_ms=self.timeout_ms, stream=stream)
+        R, cws = c.caqr_combine(gather, self.world, stream=stream)
+        (stream if stream is not None else torch.cuda.current_stream()).synchronize()
+        st = int(self.status.item())
+        if st:
+            raise c.CaqrError("caqr_peer_exchange", st)
+        return R, ws, gather, cws
+
+    def form_q(self, A_local, ws, gather, cws, opts=None, stream=None):
+        return local_form_q(A_local, ws, gather, cws, self.rank, self.world, opts=opts, stream=stream)
+
+    def close(self):
+        for p in getattr(self, "opened", []):
+            try:
+                self.caqr.caqr_ipc_close(p)
+            except Exception:
+                pass
+        self.opened = []

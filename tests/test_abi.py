@@ -98,6 +98,21 @@ def test_info_codes_without_gpu(L):
     assert c(0, 4, vp(8), 4, vp(8), 4, vp(8), 1 << 20, null) == -1
     assert c(2, 300, vp(8), 600, vp(8), 300, vp(8), 1 << 30, null) == -2
     assert L.caqr_strerror(-3) and L.caqr_strerror(1)
+    # peer-memory R exchange (alternative to the NCCL all-gather)
+    assert L.caqr_peer_mailbox_bytes(8, 192, caqr.CAQR_F32) == 2 * 8 * 192 * 192 * 4
+    assert L.caqr_peer_mailbox_bytes(0, 192, caqr.CAQR_F32) == 0
+    pe = L.caqr_peer_exchange_f32
+    assert pe(0, 0, 8, vp(8), 8, vp(8), vp(8), vp(8), 1, null, 0, null) == -1
+    assert pe(2, 2, 8, vp(8), 8, vp(8), vp(8), vp(8), 1, null, 0, null) == -2
+    assert pe(2, 0, 300, vp(8), 300, vp(8), vp(8), vp(8), 1, null, 0, null) == -3
+    assert pe(2, 0, 8, null, 8, vp(8), vp(8), vp(8), 1, null, 0, null) == -4
+    assert pe(2, 0, 8, vp(8), 4, vp(8), vp(8), vp(8), 1, null, 0, null) == -5
+    assert pe(2, 0, 8, vp(8), 8, null, vp(8), vp(8), 1, null, 0, null) == -6
+    assert pe(2, 0, 8, vp(8), 8, vp(8), null, vp(8), 1, null, 0, null) == -7
+    assert pe(2, 0, 8, vp(8), 8, vp(8), vp(8), null, 1, null, 0, null) == -8
+    assert pe(2, 0, 8, vp(8), 8, vp(8), vp(8), vp(8), 0, null, 0, null) == -9
+    assert pe(2, 0, 0, vp(8), 8, vp(8), vp(8), vp(8), 1, null, 0, null) == 0
+    assert L.caqr_ipc_handle(null, vp(8)) == -1 and L.caqr_ipc_open(null, ctypes.byref(vp())) == -1
 
 
 def test_info_codes_application_layer_without_gpu(L):

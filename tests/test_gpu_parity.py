@@ -914,3 +914,65 @@ def test_tune_info_codes(caqr):
     assert L.caqr_tune(8, 4, 7, None, 8, 1, ctypes.byref(best), ctypes.byref(f), None, None, None) == -3
     assert L.caqr_tune(8, 4, 0, None, 8, 1, ctypes.byref(best), ctypes.byref(f), None, None, None) == -4
     assert L.caqr_tune(8, 4, 0, None, 8, 1, None, ctypes.byref(f), None, None, None) == -7
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("P,m,n,dtype", [(2, 4000, 64, np.float32), (3, 9000, 100, np.float32),
+                                         (8, 16000, 192, np.float32), (3, 6000, 50, np.float64)])
+def test_peer_exchange_emulated_ranks(caqr, P, m, n, dtype):
+    """caqr_peer_exchange (the NVLink peer-store exchange, alternative to the NCCL
+    all-gather) with P virtual ranks on one device (one cooperative launch, the
+    kernel code of the per-rank call): every rank's stack must hold all P local
+    R's in rank order bit for bit, for two consecutive epochs (both mailbox
+    buffers), and the combine of any rank's stack must give the oracle's R of
+    the whole matrix (DistTSQR's result)."""
+    from paper_conf_ipps_andersonbdk11_b200 import dist as cdist
+
+    tdt = torch.float32 if dtype == np.float32 else torch.float64
+    code = caqr.CAQR_F32 if dtype == np.float32 else caqr.CAQR_F64
+    bd = BOUNDS[dtype]
+    mb_bytes = caqr.caqr_peer_mailbox_bytes(P, n, code)
+    assert mb_bytes == 2 * P * n * n * np.dtype(dtype).itemsize
+    mailboxes = [torch.full((mb_bytes // np.dtype(dtype).itemsize,), float("nan"), dtype=tdt, device="cuda")
+                 for _ in range(P)]
+    flags = [torch.zeros(P, dtype=torch.int32, device="cuda") for _ in range(P)]
+    for epoch, seed in ((1, 200 + P), (2, 300 + P)):
+        A = workloads.gaussian(m, n, seed=seed, dtype=dtype)
+        Rs = []
+        for p in range(P):
+            s0, rows = cdist.shard_rows(m, P, p)
+            Ap = caqr.colmajor_empty(rows, n, tdt)
+            Ap.copy_(torch.from_numpy(A[s0:s0 + rows]))
+            Rp, _ = caqr.caqr_factor(Ap)
+            Rs.append(Rp)
+        gathers = [caqr.colmajor_empty(P * n, n, tdt) for _ in range(P)]
+        caqr.caqr_peer_exchange_emulate(Rs, mailboxes, flags, gathers, epoch)
+        torch.cuda.synchronize()
+        want = torch.cat([r for r in Rs], dim=0)  # (P n) x n stack in rank order
+        for p in range(P):
+            assert torch.equal(gathers[p], want), (epoch, p)
+            assert torch.all(flags[p] == epoch)
+        R, _ = caqr.caqr_combine(gathers[P - 1], P)
+        torch.cuda.synchronize()
+        Rn = R.cpu().double().numpy()
+        Ro = oracle.normalize_signs(oracle.qr(A.astype(np.float64), want_q=False, acc=bd["acc"]))
+        assert np.linalg.norm(oracle.normalize_signs(Rn) - Ro) / np.linalg.norm(Ro) <= bd["r"]
+
+
+@pytest.mark.gpu
+def test_peer_exchange_arguments(caqr):
+    """Argument checks of the per-rank call (no launch on a bad argument)."""
+    R = caqr.colmajor_empty(8, 8, torch.float32)
+    g = caqr.colmajor_empty(16, 8, torch.float32)
+    ptrs = torch.zeros(2, dtype=torch.int64, device="cuda")
+    L = caqr.lib()
+    assert L.caqr_peer_exchange_f32(0, 0, 8, R.data_ptr(), 8, ptrs.data_ptr(), ptrs.data_ptr(), g.data_ptr(),
+                                    1, None, 0, None) == -1
+    assert L.caqr_peer_exchange_f32(2, 2, 8, R.data_ptr(), 8, ptrs.data_ptr(), ptrs.data_ptr(), g.data_ptr(),
+                                    1, None, 0, None) == -2
+    assert L.caqr_peer_exchange_f32(2, 0, 8, R.data_ptr(), 4, ptrs.data_ptr(), ptrs.data_ptr(), g.data_ptr(),
+                                    1, None, 0, None) == -5
+    assert L.caqr_peer_exchange_f32(2, 0, 8, R.data_ptr(), 8, ptrs.data_ptr(), ptrs.data_ptr(), g.data_ptr(),
+                                    0, None, 0, None) == -9
+    assert L.caqr_peer_exchange_f32(2, 0, 0, R.data_ptr(), 8, ptrs.data_ptr(), ptrs.data_ptr(), g.data_ptr(),
+                                    1, None, 0, None) == 0
