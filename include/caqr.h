@@ -393,6 +393,31 @@ int caqr_rpca_update_f32(int64_t m, int64_t n, const float *M, int64_t ldm, cons
 int caqr_rpca_init_f32(int64_t m, int64_t n, const float *M, int64_t ldm, float yscale, float *S,
                        int64_t lds, float *Y, int64_t ldy, float *X, int64_t ldx, float mu,
                        caqr_stream_t stream);
+/* The iteration's scalar schedule on the device (reading S19 of DESIGN.md), so
+ * that no step needs a host round trip: sched (device double[CAQR_RPCA_SCHED_LEN])
+ * <- mu = mu_factor / sigma[0] (||M||_2 from the QR + small SVD of M), mu_max =
+ * mu_max_factor mu, rho, yscale = 1 / max(sigma[0], amax[0] / lambda)
+ * (||M||_inf from caqr_absmax_f32), lambda.  The *_sched_f32 variants of
+ * rpca_init / svt_core_r / rpca_update read their scalars from it (in double,
+ * converted as the by-value entry points receive them), and rpca_update_sched
+ * advances mu <- min(rho mu, mu_max) after its pass (stream order).
+ * info: -1 sigma, -2 amax, -3 lambda <= 0, -4 mu_factor <= 0,
+ * -5 mu_max_factor < 1, -6 rho < 1, -7 sched. */
+#define CAQR_RPCA_SCHED_LEN 8
+int caqr_rpca_schedule_f32(const float *sigma, const float *amax, double lambda, double mu_factor,
+                           double mu_max_factor, double rho, double *sched, caqr_stream_t stream);
+/* caqr_rpca_init_f32 with yscale and mu from sched.  info as caqr_rpca_init_f32 with
+ * -5 = sched. */
+int caqr_rpca_init_sched_f32(int64_t m, int64_t n, const float *M, int64_t ldm, const double *sched, float *S,
+                             int64_t lds, float *Y, int64_t ldy, float *X, int64_t ldx, caqr_stream_t stream);
+/* caqr_svt_core_r_f32 with tau = 1 / sched[0].  info: -7 sched, otherwise as caqr_svt_core_r_f32. */
+int caqr_svt_core_r_sched_f32(int64_t n, const float *U, int64_t ldu, const float *sigma, const float *R,
+                              int64_t ldr, const double *sched, float *W, int64_t ldw, caqr_stream_t stream);
+/* caqr_rpca_update_f32 with mu = sched[0], mu_next = min(rho mu, mu_max), lambda from sched;
+ * sched[0] <- mu_next afterwards.  info: -13 sched, -14 resid, otherwise as caqr_rpca_update_f32. */
+int caqr_rpca_update_sched_f32(int64_t m, int64_t n, const float *M, int64_t ldm, const float *L, int64_t ldl,
+                               float *S, int64_t lds, float *Y, int64_t ldy, float *X, int64_t ldx, double *sched,
+                               double *resid, caqr_stream_t stream);
 /* out[0] (device float) = max |M_ij| (0 for an empty M).  info: -1 m, -2 n, -3 M, -4 ldm, -5 out. */
 int caqr_absmax_f32(int64_t m, int64_t n, const float *M, int64_t ldm, float *out, caqr_stream_t stream);
 

@@ -150,7 +150,14 @@ def lib() -> ctypes.CDLL:
                                            vp, vp]
         L.caqr_rpca_init_f32.argtypes = [i64, i64, vp, i64, fl, vp, i64, vp, i64, vp, i64, fl, vp]
         L.caqr_absmax_f32.argtypes = [i64, i64, vp, i64, vp, vp]
-        for name in ("svt_core", "svt_core_r", "embed_top", "rpca_update", "rpca_init", "absmax"):
+        db = ctypes.c_double
+        L.caqr_rpca_schedule_f32.argtypes = [vp, vp, db, db, db, db, vp, vp]
+        L.caqr_rpca_init_sched_f32.argtypes = [i64, i64, vp, i64, vp, vp, i64, vp, i64, vp, i64, vp]
+        L.caqr_svt_core_r_sched_f32.argtypes = [i64, vp, i64, vp, vp, i64, vp, vp, i64, vp]
+        L.caqr_rpca_update_sched_f32.argtypes = [i64, i64, vp, i64, vp, i64, vp, i64, vp, i64, vp, i64, vp, vp,
+                                                 vp]
+        for name in ("svt_core", "svt_core_r", "embed_top", "rpca_update", "rpca_init", "absmax", "rpca_schedule",
+                     "rpca_init_sched", "svt_core_r_sched", "rpca_update_sched"):
             getattr(L, f"caqr_{name}_f32").restype = ip
         _lib = L
         return L
@@ -584,6 +591,48 @@ def caqr_rpca_init(M, yscale: float, S, Y, X, mu: float, stream=None):
     px, ldx = _f32(X, "X")
     _check("caqr_rpca_init_f32", lib().caqr_rpca_init_f32(m, n, pm, ldm, float(yscale), ps, lds, py, ldy, px, ldx,
                                                           float(mu), _stream(stream)))
+
+
+CAQR_RPCA_SCHED_LEN = 8
+
+
+def caqr_rpca_schedule(sigma, amax, lam: float, mu_factor: float, mu_max_factor: float, rho: float, sched,
+                       stream=None):
+    """sched (device float64[8]) <- mu, mu_max, rho, yscale, lambda from sigma[0] and amax[0]."""
+    _check("caqr_rpca_schedule_f32", lib().caqr_rpca_schedule_f32(sigma.data_ptr(), amax.data_ptr(), float(lam),
+                                                                  float(mu_factor), float(mu_max_factor),
+                                                                  float(rho), sched.data_ptr(), _stream(stream)))
+    return sched
+
+
+def caqr_rpca_init_sched(M, sched, S, Y, X, stream=None):
+    m, n = M.shape
+    pm, ldm = _f32(M, "M")
+    ps, lds = _f32(S, "S")
+    py, ldy = _f32(Y, "Y")
+    px, ldx = _f32(X, "X")
+    _check("caqr_rpca_init_sched_f32", lib().caqr_rpca_init_sched_f32(m, n, pm, ldm, sched.data_ptr(), ps, lds, py,
+                                                                      ldy, px, ldx, _stream(stream)))
+
+
+def caqr_svt_core_r_sched(U, sigma, R, sched, W=None, stream=None):
+    n = U.shape[0]
+    pu, ldu = _f32(U, "U")
+    pr, ldr = _f32(R, "R")
+    W = colmajor_empty(n, n, U.dtype, U.device) if W is None else W
+    pw, ldw = _f32(W, "W")
+    _check("caqr_svt_core_r_sched_f32", lib().caqr_svt_core_r_sched_f32(n, pu, ldu, sigma.data_ptr(), pr, ldr,
+                                                                        sched.data_ptr(), pw, ldw, _stream(stream)))
+    return W
+
+
+def caqr_rpca_update_sched(M, L, S, Y, X, sched, resid, stream=None):
+    m, n = M.shape
+    args = []
+    for t, nm in ((M, "M"), (L, "L"), (S, "S"), (Y, "Y"), (X, "X")):
+        args += list(_f32(t, nm))
+    _check("caqr_rpca_update_sched_f32", lib().caqr_rpca_update_sched_f32(m, n, *args, sched.data_ptr(),
+                                                                          resid.data_ptr(), _stream(stream)))
 
 
 def caqr_absmax(M, out, stream=None):

@@ -1856,6 +1856,90 @@ int caqr_rpca_init_f32(int64_t m, int64_t n, const float* M, int64_t ldm, float 
     return launch_status();
 }
 
+int caqr_rpca_schedule_f32(const float* sigma, const float* amax, double lambda, double mu_factor,
+                           double mu_max_factor, double rho, double* sched, caqr_stream_t stream) {
+    if (!sigma) return -1;
+    if (!amax) return -2;
+    if (!(lambda > 0.0)) return -3;
+    if (!(mu_factor > 0.0)) return -4;
+    if (!(mu_max_factor >= 1.0)) return -5;
+    if (!(rho >= 1.0)) return -6;
+    if (!sched) return -7;
+    rpca_schedule_kernel<<<1, 32, 0, (cudaStream_t)stream>>>(sigma, amax, lambda, mu_factor, mu_max_factor, rho,
+                                                             sched);
+    return launch_status();
+}
+
+int caqr_rpca_init_sched_f32(int64_t m, int64_t n, const float* M, int64_t ldm, const double* sched, float* S,
+                             int64_t lds, float* Y, int64_t ldy, float* X, int64_t ldx, caqr_stream_t stream) {
+    if (m < 0) return -1;
+    if (n < 0) return -2;
+    const int64_t lm = std::max<int64_t>(1, m);
+    if (ldm < lm) return -4;
+    if (!sched) return -5;
+    if (lds < lm) return -7;
+    if (ldy < lm) return -9;
+    if (ldx < lm) return -11;
+    if (m == 0 || n == 0) return 0;
+    if (!M) return -3;
+    if (!S) return -6;
+    if (!Y) return -8;
+    if (!X) return -10;
+    cudaStream_t s = (cudaStream_t)stream;
+    TraceScope ts(K_RPCA_INIT, 2.0 * m * n, 4.0 * 4 * m * n, s);
+    rpca_init_kernel<float><<<elem_grid(m * n, 256), 256, 0, s>>>(m, n, M, ldm, 0.f, S, lds, Y, ldy, X, ldx, 1.f,
+                                                                  sched);
+    return launch_status();
+}
+
+int caqr_svt_core_r_sched_f32(int64_t n, const float* U, int64_t ldu, const float* sigma, const float* R,
+                              int64_t ldr, const double* sched, float* W, int64_t ldw, caqr_stream_t stream) {
+    if (n < 0 || n > kSvdMaxN) return -1;
+    if (ldu < std::max<int64_t>(1, n)) return -3;
+    if (ldr < std::max<int64_t>(1, n)) return -6;
+    if (!sched) return -7;
+    if (ldw < std::max<int64_t>(1, n)) return -9;
+    if (n == 0) return 0;
+    if (!U) return -2;
+    if (!sigma) return -4;
+    if (!R) return -5;
+    if (!W) return -8;
+    cudaStream_t s = (cudaStream_t)stream;
+    TraceScope ts(K_SVT_CORE, 4.0 * n * n * n, 4.0 * 3 * n * n, s);
+    svt_core_r_kernel<float><<<(unsigned)n, 128, 0, s>>>((int)n, U, ldu, sigma, R, ldr, 0.f, W, ldw, sched);
+    return launch_status();
+}
+
+int caqr_rpca_update_sched_f32(int64_t m, int64_t n, const float* M, int64_t ldm, const float* L, int64_t ldl,
+                               float* S, int64_t lds, float* Y, int64_t ldy, float* X, int64_t ldx, double* sched,
+                               double* resid, caqr_stream_t stream) {
+    if (m < 0) return -1;
+    if (n < 0) return -2;
+    const int64_t lm = std::max<int64_t>(1, m);
+    if (ldm < lm) return -4;
+    if (ldl < lm) return -6;
+    if (lds < lm) return -8;
+    if (ldy < lm) return -10;
+    if (ldx < lm) return -12;
+    if (!sched) return -13;
+    if (!resid) return -14;
+    if (m > 0 && n > 0) {
+        if (!M) return -3;
+        if (!L) return -5;
+        if (!S) return -7;
+        if (!Y) return -9;
+        if (!X) return -11;
+    }
+    cudaStream_t s = (cudaStream_t)stream;
+    {
+        TraceScope ts(K_RPCA_UPDATE, 12.0 * m * n, 4.0 * 7 * m * n, s);
+        rpca_update_kernel<float><<<kRpcaBlocks, 256, 0, s>>>(m, n, M, ldm, L, ldl, S, lds, Y, ldy, X, ldx, 1.f, 1.f,
+                                                              0.f, resid, sched);
+    }
+    sum_parts_kernel<<<1, 256, 0, s>>>(kRpcaBlocks, resid, sched);  // also mu <- min(rho mu, mu_max)
+    return launch_status();
+}
+
 int caqr_absmax_f32(int64_t m, int64_t n, const float* M, int64_t ldm, float* out, caqr_stream_t stream) {
     if (m < 0) return -1;
     if (n < 0) return -2;

@@ -359,8 +359,10 @@ __global__ void svt_core_kernel(int n, const T* __restrict__ U, int64_t ldu, con
 // sigma_j > tau, hence no small sigma, is divided by).  One block per column k.
 template <typename T>
 __global__ void svt_core_r_kernel(int n, const T* __restrict__ U, int64_t ldu, const T* __restrict__ sigma,
-                                  const T* __restrict__ R, int64_t ldr, T tau, T* __restrict__ W, int64_t ldw) {
+                                  const T* __restrict__ R, int64_t ldr, T tau, T* __restrict__ W, int64_t ldw,
+                                  const double* __restrict__ sched = nullptr) {
     __shared__ double pk[kSvdMaxN];
+    if (sched) tau = (T)(1.0 / sched[0]);  // the iteration's 1/mu (device schedule)
     const int k = blockIdx.x;
     for (int j = threadIdx.x; j < n; j += blockDim.x) {  // pk_j = f(sigma_j) (U^T R)_jk
         const double sj = (double)sigma[j], d = sj - (double)tau;
@@ -409,8 +411,14 @@ __global__ void __launch_bounds__(256) rpca_update_kernel(int64_t m, int64_t n, 
                                                           const T* __restrict__ L, int64_t ldl, T* __restrict__ S,
                                                           int64_t lds, T* __restrict__ Y, int64_t ldy,
                                                           T* __restrict__ X, int64_t ldx, T mu, T mu_next,
-                                                          T lambda, double* __restrict__ part) {
+                                                          T lambda, double* __restrict__ part,
+                                                          const double* __restrict__ sched = nullptr) {
     __shared__ double scr[8];
+    if (sched) {  // device schedule: mu, mu_next = min(rho mu, mu_max), lambda
+        mu = (T)sched[0];
+        mu_next = (T)fmin(sched[2] * sched[0], sched[1]);
+        lambda = (T)sched[4];
+    }
     const T imu = T(1) / mu, imu_next = T(1) / mu_next, thr = lambda / mu;
     double acc = 0.0;
     const int64_t total = m * n;
@@ -432,20 +440,45 @@ __global__ void __launch_bounds__(256) rpca_update_kernel(int64_t m, int64_t n, 
 }
 
 // part[0] = sum of part[1..nb] in index order (deterministic).
-__global__ void sum_parts_kernel(int nb, double* part) {
+// With a device schedule it also advances mu <- min(rho mu, mu_max) (this
+// kernel runs after the update kernel that read mu, on the same stream).
+__global__ void sum_parts_kernel(int nb, double* part, double* sched = nullptr) {
     __shared__ double scr[32];
     double a = 0.0;
     // fixed assignment of parts to threads and a fixed tree: deterministic
     for (int b = threadIdx.x; b < nb; b += blockDim.x) a += part[1 + b];
     const double t = block_sum_d(a, scr);
-    if (threadIdx.x == 0) part[0] = t;
+    if (threadIdx.x == 0) {
+        part[0] = t;
+        if (sched) sched[0] = fmin(sched[2] * sched[0], sched[1]);
+    }
+}
+
+// Device schedule of the iteration (reading S19): from ||M||_2 = sigma[0] and
+// ||M||_inf = amax[0]: mu0 = mu_factor / ||M||_2, mu_max = mu_max_factor mu0,
+// rho, yscale = 1 / max(||M||_2, ||M||_inf / lambda), lambda -- in double.
+__global__ void rpca_schedule_kernel(const float* __restrict__ sigma, const float* __restrict__ amax, double lambda,
+                                     double mu_factor, double mu_max_factor, double rho, double* sched) {
+    if (threadIdx.x != 0) return;
+    const double norm2 = (double)sigma[0], norminf = (double)amax[0];
+    const double J = fmax(norm2, norminf / lambda);
+    const double mu = mu_factor / norm2;
+    sched[0] = mu;
+    sched[1] = mu * mu_max_factor;
+    sched[2] = rho;
+    sched[3] = 1.0 / J;
+    sched[4] = lambda;
 }
 
 // Start of the iteration: S = 0, Y = yscale M, X = M + Y / mu.
 template <typename T>
 __global__ void rpca_init_kernel(int64_t m, int64_t n, const T* __restrict__ M, int64_t ldm, T yscale,
                                  T* __restrict__ S, int64_t lds, T* __restrict__ Y, int64_t ldy, T* __restrict__ X,
-                                 int64_t ldx, T mu) {
+                                 int64_t ldx, T mu, const double* __restrict__ sched = nullptr) {
+    if (sched) {
+        yscale = (T)sched[3];
+        mu = (T)sched[0];
+    }
     const int64_t total = m * n;
     const T imu = T(1) / mu;
     for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {

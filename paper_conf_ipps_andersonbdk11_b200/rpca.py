@@ -15,8 +15,9 @@ reading S19).  Every iteration:
   5. S = shrink(M - L + Y/mu, lambda/mu); Y += mu (M - L - S); the next X
      (caqr_rpca_update_f32, one fused pass)
 
-This module only allocates buffers and keeps the scalar schedule (mu); every
-arithmetic step is a libcaqr kernel.  There is no CPU path.
+This module only allocates buffers; every arithmetic step, the scalar schedule
+(mu, mu_max, rho, lambda: caqr_rpca_schedule_f32 and the *_sched_f32 kernels)
+included, runs in libcaqr on the device.  There is no CPU path.
 """
 from __future__ import annotations
 
@@ -46,20 +47,36 @@ class RobustPCA:
                               device=dev)
         self.resid = torch.zeros(caqr.CAQR_RPCA_RESID_LEN, dtype=torch.float64, device=dev)
         self.amax = torch.zeros(1, dtype=torch.float32, device=dev)
-        self.lam = 1.0 / math.sqrt(max(m, n))
-        self.rho = rho
+        # the scalar schedule lives on the device (mu, mu_max, rho, yscale, lambda):
+        # no step needs a host round trip
+        self.sched = torch.zeros(caqr.CAQR_RPCA_SCHED_LEN, dtype=torch.float64, device=dev)
         # ||M||_2 through the same QR + small SVD, ||M||_inf by a max reduction
         self.X.copy_(self.M)
         caqr.caqr_factor(self.X, R=self.R, ws=self.ws, opts=opts, stream=stream)
         caqr.caqr_svd_small(self.R, self.U, self.sigma, stream=stream, want_v=False)
         caqr.caqr_absmax(self.M, self.amax, stream=stream)
-        norm2 = float(self.sigma[0].item())
-        norminf = float(self.amax[0].item())
-        J = max(norm2, norminf / self.lam)
-        self.mu = mu_factor / norm2
-        self.mu_max = self.mu * mu_max_factor
-        caqr.caqr_rpca_init(self.M, 1.0 / J, self.S, self.Y, self.X, self.mu, stream=stream)
+        caqr.caqr_rpca_schedule(self.sigma, self.amax, 1.0 / math.sqrt(max(m, n)), mu_factor, mu_max_factor, rho,
+                                self.sched, stream=stream)
+        caqr.caqr_rpca_init_sched(self.M, self.sched, self.S, self.Y, self.X, stream=stream)
         self.iters = 0
+
+    # schedule entries (reading them synchronises; setting them is a device write)
+    def _get(self, i: int) -> float:
+        import torch
+
+        (self.stream or torch.cuda.current_stream()).synchronize()
+        return float(self.sched[i].item())
+
+    def _set(self, i: int, v: float):
+        import torch
+
+        with torch.cuda.stream(self.stream or torch.cuda.current_stream()):
+            self.sched[i:i + 1].fill_(float(v))
+
+    mu = property(lambda self: self._get(0), lambda self, v: self._set(0, v))
+    mu_max = property(lambda self: self._get(1), lambda self, v: self._set(1, v))
+    rho = property(lambda self: self._get(2), lambda self, v: self._set(2, v))
+    lam = property(lambda self: self._get(4), lambda self, v: self._set(4, v))
 
     def load_state(self, S, Y, X, mu: float):
         """Set the iteration state (S, Y, the SVT input X = M - S + Y/mu, mu):
@@ -67,20 +84,17 @@ class RobustPCA:
         self.S.copy_(S)
         self.Y.copy_(Y)
         self.X.copy_(X)
-        self.mu = float(mu)
+        self.mu = mu
 
     def step(self):
-        """One iteration; returns nothing (no host synchronisation)."""
+        """One iteration; returns nothing (no host synchronisation, no host scalar)."""
         s, o = self.stream, self.opts
         caqr.caqr_factor(self.X, R=self.R, ws=self.ws, opts=o, stream=s)
         caqr.caqr_svd_small(self.R, self.U, self.sigma, stream=s, want_v=False)
-        caqr.caqr_svt_core_r(self.U, self.sigma, self.R, 1.0 / self.mu, self.W, stream=s)
+        caqr.caqr_svt_core_r_sched(self.U, self.sigma, self.R, self.sched, self.W, stream=s)
         caqr.caqr_embed_top(self.W, self.L, stream=s)
         caqr.caqr_apply_q(self.X, self.ws, self.L, opts=o, stream=s)
-        mu_next = min(self.rho * self.mu, self.mu_max)
-        caqr.caqr_rpca_update(self.M, self.L, self.S, self.Y, self.X, self.mu, mu_next, self.lam, self.resid,
-                              stream=s)
-        self.mu = mu_next
+        caqr.caqr_rpca_update_sched(self.M, self.L, self.S, self.Y, self.X, self.sched, self.resid, stream=s)
         self.iters += 1
 
     def residual(self) -> float:
