@@ -23,11 +23,21 @@ def run(m, n, dt=torch.float32, opts=None):
 which = sys.argv[1] if len(sys.argv) > 1 else "all"
 if which in ("all", "fused"):
     run(20000, 48)                     # fused, chains + tree
+    run(30000, 100)                    # fused: 4 panels, ragged last (4 columns), 3-block trailing updates
     run(5000, 40, torch.float64)       # fused fp64
 if which in ("all", "stream"):
     run(300_000, 8)                    # streaming skinny kernel
 if which in ("all", "caqr"):
     run(600, 300, opts=caqr.make_opts(panel_cols=64))  # CAQR panel loop (split + early start)
+if which in ("all", "peer"):
+    P, n = 3, 24
+    Rs = [torch.triu(torch.randn(n, n, device="cuda")).t().contiguous().t() for _ in range(P)]
+    mb = [torch.zeros(caqr.caqr_peer_mailbox_bytes(P, n, caqr.CAQR_F32) // 4, device="cuda") for _ in range(P)]
+    fl = [torch.zeros(P, dtype=torch.int32, device="cuda") for _ in range(P)]
+    for ep in (1, 2):
+        gs = [caqr.colmajor_empty(P * n, n) for _ in range(P)]
+        caqr.caqr_peer_exchange_emulate(Rs, mb, fl, gs, ep)
+    torch.cuda.synchronize()
 if which in ("all", "rpca"):
     M = workloads.video(frames=20, h=48, w=64).astype(np.float32)
     Md = caqr.colmajor_empty(*M.shape)
