@@ -148,7 +148,14 @@ static int make_plan(int64_t m, int64_t n, int dtype, const caqr_opts* o, int op
     int64_t b = (o && o->leaf_rows > 0) ? o->leaf_rows
                                         : pl->chain ? chain_tile_rows(n)
                                         : (pl->skinny ? (n <= 8 && !s16 ? 256 : 128)
-                                                      : (nb <= kFusedLeaf && n <= 224 ? kFusedLeaf : kMaxLeaf));
+                                                      : (nb <= kFusedLeaf && (n <= 224 || ceil_div(m, kMaxLeaf) >
+                                                                                              pl->chain_target)
+                                                             ? kFusedLeaf
+                                                             : kMaxLeaf));
+    // (256-row tiles only when every chain is one tile: a chain step of a
+    // 256-row tile gathers 288 rows, beyond the fused kernel, so tall groups
+    // of a 224 < n <= 256 matrix would fall back to the split path --
+    // measured 1M x 256: 31.6 ms with b = 256 vs 1M x 192: 5.3 ms)
     if (b % 32 != 0 || b > kMaxLeaf) return -opt_pos;
     b = std::max(b, round_up(nb, 32));
     if (b > kMaxLeaf) return -opt_pos;

@@ -119,6 +119,18 @@ def test_factor_parity(caqr, shape, dtype):
     check_against_oracle(caqr, A)
 
 
+@pytest.mark.parametrize("shape", [(90000, 256), (80000, 232)], ids=lambda s: f"{s[0]}x{s[1]}")
+def test_tall_wide_groups_parity(caqr, shape):
+    """Tall matrices with 224 < n <= 256: two 128-column panel groups of
+    224-row tiles in chains (the fused kernel for both groups' TSQRs, the
+    tree-replayed trailing update between them), against the oracle at the
+    unrelaxed bounds of check_against_oracle."""
+    info = caqr.caqr_plan_info(*shape)
+    assert info["groups"] == 2 and info["leaf_rows"] == 224 and info["leaves"] > info["chains"]
+    A = workloads.gaussian(*shape, seed=shape[1] + 11)
+    check_against_oracle(caqr, A)
+
+
 @pytest.mark.parametrize("leaf_rows", [32, 64, 128, 256])
 def test_leaf_size_sweep(caqr, leaf_rows):
     """Uniqueness of R: every leaf size / tree gives the oracle's R (S5, S6)."""
