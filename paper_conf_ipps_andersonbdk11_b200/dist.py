@@ -238,6 +238,8 @@ class PeerTSQR:
         Rl, ws = c.caqr_factor(A_local, opts=opts, stream=stream)
         self.epoch += 1
         gather = c.colmajor_empty(self.world * n, n, A_local.dtype, A_local.device)
+        with torch.cuda.stream(stream or torch.cuda.current_stream()):
+            self.status.zero_()  # a previous call's timeout must not fail this one
         c.caqr_peer_exchange(self.world, self.rank, Rl, self.mb_ptrs, self.fl_ptrs, gather, self.epoch,
                              status=self.status, timeout_ms=self.timeout_ms, stream=stream)
         R, cws = c.caqr_combine(gather, self.world, stream=stream)
