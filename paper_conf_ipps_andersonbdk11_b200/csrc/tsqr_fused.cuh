@@ -3,9 +3,10 @@
 // Every tree node -- leaf row block ("factor") or merge of two R
 // factors ("factor_tree") -- is one task for one CTA.  A task walks
 // its <=32-column panels: stage the gathered rows of panel p in shared memory,
-// factor it with the panel held in registers (8 threads per column, one CTA
-// barrier per column: matvec + rank-1 update of P:L704-711), write R / V and the
-// compact-WY T, then apply (I - V T V^T)^T to the node's trailing
+// factor it with the panel held in registers (factor_panel_pipe: each warp owns
+// 4 columns, reflectors published one by one through shared-memory mbarriers:
+// matvec + rank-1 update of P:L704-711), write R / V and the compact-WY T
+// (P:L224-246), then apply (I - V T V^T)^T to the node's trailing
 // columns block by block (the horizontal update of P:L665-668 done inside the
 // node) and publish "slot s, panel p done".  Tasks are handed out by an atomic
 // ticket in topological order (leaves, then tree level by level); a merge waits
@@ -19,7 +20,7 @@
 namespace caqr {
 
 // Row index of a shared panel / C tile.  Plain (identity): every access pattern
-// that remains is conflict-free without row padding -- WB4 and the staging /
+// that remains is conflict-free without row padding -- the panel and the staging /
 // write-back loops have lanes on consecutive rows, and the GEMM fragments
 // differ by column, which the column stride (16 bytes mod 128) spreads over
 // the banks.  (An earlier 8-threads-per-column panel layout needed padding
