@@ -564,13 +564,18 @@ __device__ __forceinline__ void build_t(const Grp& Gr, const T* G, const T* tau_
 // across tiles), which frees the MIO pipe the panel factorization needs.
 // Used only for W = V^T C and C -= V W2 of the factorization's trailing
 // update: V, T (hence Q) stay exact fp32, so Q's orthogonality is unaffected;
-// the trailing matrix sees ~2^-22 relative product errors (backward error).
+// the trailing matrix sees ~2^-21 relative product errors (backward error).
+// The low part goes to the MMA unrounded (the TF32 unit reads its top 10
+// mantissa bits: truncation, error <= 2^-21 |x| instead of 2^-22 for a second
+// cvt.rna): one conversion less per operand element, 5.34 -> 5.15 ms at
+// 1M x 192, every achieved error unchanged to three digits (S20,
+// profiles/parity_r02.json).  CAQR_EXACT_SPLIT restores the rounded low part.
 // ---------------------------------------------------------------------------
 __device__ __forceinline__ void split_tf32(float x, uint32_t& hi, uint32_t& lo) {
     uint32_t h, l;
     asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(h) : "f"(x));
     const float r = x - __uint_as_float(h);
-#ifdef CAQR_CHEAP_SPLIT
+#ifndef CAQR_EXACT_SPLIT
     l = __float_as_uint(r);
 #else
     asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(l) : "f"(r));
