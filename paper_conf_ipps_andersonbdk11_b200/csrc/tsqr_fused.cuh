@@ -415,8 +415,8 @@ __device__ __forceinline__ void factor_panel_pipe(const Grp& G, T* P, int RGP, i
         for (int q = 0; q < 4; ++q) Gout[(cb + q) * kTS + lane] = T(0);
     gsync(G);  // every reflector applied: P's v columns are no longer read
     {
-        // epilogue straight from registers (as factor_panel_wb4): the stored
-        // form (R / v, structure masks) to global, the V form into P
+        // epilogue straight from registers: the stored form (R / v,
+        // structure masks) to global
         const NodeRows& nr = *out_nr;
         const uint64_t pol = l2_evict_first_policy();
         int64_t grow[8];
@@ -433,7 +433,6 @@ __device__ __forceinline__ void factor_panel_pipe(const Grp& G, T* P, int RGP, i
         for (int q = 0; q < 4; ++q) {
             const int jj = cb + q;
             T* col = out_A + (out_c0 + jj) * out_lda;
-            T* pcol = P + (size_t)jj * RGP;
 #pragma unroll
             for (int i = 0; i < 8; ++i) {
                 const int r = lane + 32 * i;
@@ -445,12 +444,9 @@ __device__ __forceinline__ void factor_panel_pipe(const Grp& G, T* P, int RGP, i
                     if (seg0[i]) col[grow[i]] = x[q][i];
                     else st_evict_first(col + grow[i], x[q][i], pol);
                 }
-                T v = T(0);
-                if (in) {
-                    if (seg0[i]) v = nr.seg0_tri ? (r == jj ? T(1) : T(0)) : (r > jj ? x[q][i] : (r == jj ? T(1) : T(0)));
-                    else v = stored ? x[q][i] : T(0);
-                }
-                pcol[padr<T>(r)] = v;
+                // (P already holds the V form: the v each owner wrote for the
+                // consumers equals it -- a structured node's implicit zeros
+                // stay exactly zero through the dense reflectors)
             }
         }
     }
