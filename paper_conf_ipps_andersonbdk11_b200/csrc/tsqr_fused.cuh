@@ -414,10 +414,34 @@ __device__ __forceinline__ void factor_panel_pipe(const Grp& G, T* P, int RGP, i
 #pragma unroll
         for (int q = 0; q < 4; ++q) Gout[(cb + q) * kTS + lane] = T(0);
     gsync(G);  // every reflector applied: P's v columns are no longer read
-    {
+    const NodeRows& nr = *out_nr;
+    if (!nr.seg1_upper && (nr.n1 == 0 || (nr.seg0_tri && nr.n0 == 32))) {
+        // fast epilogue for the two common node shapes (warp-uniform test):
+        // a leaf (one dense segment, everything stored) and a full chain step
+        // (gathered rows 0..31 = the R band, stored on and above the
+        // diagonal; rows 32.. = the tile, dense, final V)
+        const uint64_t pol = l2_evict_first_policy();
+        const bool leaf = nr.n1 == 0;
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            if (q >= nc) continue;
+            const int jj = cb + q;
+            T* col = out_A + (out_c0 + jj) * out_lda;
+            if (leaf) {
+#pragma unroll
+                for (int i = 0; i < 8; ++i)
+                    if (lane + 32 * i < RG) col[nr.r0 + lane + 32 * i] = x[q][i];
+            } else {
+                if (lane <= jj) col[nr.r0 + lane] = x[q][0];
+                T* tcol = col + nr.r1 - 32;
+#pragma unroll
+                for (int i = 1; i < 8; ++i)
+                    if (lane + 32 * i < RG) st_evict_first(tcol + lane + 32 * i, x[q][i], pol);
+            }
+        }
+    } else {
         // epilogue straight from registers: the stored form (R / v,
         // structure masks) to global
-        const NodeRows& nr = *out_nr;
         const uint64_t pol = l2_evict_first_policy();
         int64_t grow[8];
         int key[8];
