@@ -415,13 +415,15 @@ __device__ __forceinline__ void factor_panel_pipe(const Grp& G, T* P, int RGP, i
         for (int q = 0; q < 4; ++q) Gout[(cb + q) * kTS + lane] = T(0);
     gsync(G);  // every reflector applied: P's v columns are no longer read
     const NodeRows& nr = *out_nr;
-    if (!nr.seg1_upper && (nr.n1 == 0 || (nr.seg0_tri && nr.n0 == 32))) {
-        // fast epilogue for the two common node shapes (warp-uniform test):
-        // a leaf (one dense segment, everything stored) and a full chain step
-        // (gathered rows 0..31 = the R band, stored on and above the
-        // diagonal; rows 32.. = the tile, dense, final V)
+    if ((!nr.seg1_upper && nr.n1 == 0) || (nr.seg0_tri && nr.n0 == 32)) {
+        // fast epilogue for the common node shapes (warp-uniform test): a leaf
+        // (one dense segment, everything stored), a full chain step (gathered
+        // rows 0..31 = the R band, stored on and above the diagonal; rows 32..
+        // = the tile, dense, final V) and a full merge (rows 32.. = the right
+        // member's R slot, stored on and above its diagonal: final tree V)
         const uint64_t pol = l2_evict_first_policy();
-        const bool leaf = nr.n1 == 0;
+        const bool leaf = !nr.seg1_upper && nr.n1 == 0;
+        const int upper = nr.seg1_upper ? 32 + 32 * out_p : (1 << 30);  // seg1 row r stored iff r - upper <= jj
 #pragma unroll
         for (int q = 0; q < 4; ++q) {
             if (q >= nc) continue;
@@ -436,7 +438,8 @@ __device__ __forceinline__ void factor_panel_pipe(const Grp& G, T* P, int RGP, i
                 T* tcol = col + nr.r1 - 32;
 #pragma unroll
                 for (int i = 1; i < 8; ++i)
-                    if (lane + 32 * i < RG) st_evict_first(tcol + lane + 32 * i, x[q][i], pol);
+                    if (lane + 32 * i < RG && lane + 32 * i - upper <= jj)
+                        st_evict_first(tcol + lane + 32 * i, x[q][i], pol);
             }
         }
     } else {
